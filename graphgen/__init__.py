@@ -1,0 +1,182 @@
+"""Seeded synthetic inputs for MergePath-SpMM (graphs, edge values, dense B).
+
+Used by BOTH sides of every parity check (tests, bench, smoke); holds none of the
+method's arithmetic.  The arrays come from ``graphgen/gen.cpp`` (C++17/OpenMP, built with
+g++), a counter-based generator, so a (recipe, seed) pair always yields the same
+bytes on any machine and thread count.  The recipes follow DESIGN.md "Input recipe":
+sizes and degree skew of the paper's Table II graphs and of the
+BASELINE.json configs.
+"""
+from __future__ import annotations
+
+import ctypes
+import hashlib
+import os
+import subprocess
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "gen.cpp")
+_LIB_PATH = os.path.join(_HERE, "libmpsgen.so")
+_lib = None
+_i64, _i32, _u64, _f64, _p = (ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64,
+                              ctypes.c_double, ctypes.c_void_p)
+
+
+def build(force: bool = False) -> str:
+    if (not force and os.path.exists(_LIB_PATH)
+            and os.path.getmtime(_LIB_PATH) >= os.path.getmtime(_SRC)):
+        return _LIB_PATH
+    tmp = _LIB_PATH + ".tmp%d" % os.getpid()
+    subprocess.check_call(["g++", "-std=c++17", "-O2", "-fopenmp", "-fPIC", "-shared", _SRC,
+                           "-o", tmp])
+    os.replace(tmp, _LIB_PATH)
+    return _LIB_PATH
+
+
+def _L():
+    global _lib
+    if _lib is None:
+        build()
+        lib = ctypes.CDLL(_LIB_PATH)
+        lib.gen_chung_lu.argtypes = [_i64, _i64, _f64, _f64, _u64]
+        lib.gen_chung_lu.restype = _p
+        lib.gen_rmat.argtypes = [_i32, _i64, _f64, _f64, _f64, _i32, _i64, _u64]
+        lib.gen_rmat.restype = _p
+        lib.gen_random_csr.argtypes = [_i64, _i64, _p, _i32, _u64]
+        lib.gen_random_csr.restype = _p
+        for f in ("gen_rows", "gen_cols", "gen_nnz"):
+            getattr(lib, f).argtypes = [_p]
+            getattr(lib, f).restype = _i64
+        lib.gen_copy.argtypes = [_p, _p, _p]
+        lib.gen_free.argtypes = [_p]
+        lib.gen_values_gcn.argtypes = [_i64, _p, _p, _p]
+        lib.gen_values_int.argtypes = [_i64, _u64, _p]
+        lib.gen_dense_uniform.argtypes = [_i64, _i32, _i64, _u64, _p]
+        lib.gen_dense_int.argtypes = [_i64, _i32, _i64, _u64, _p]
+        _lib = lib
+    return _lib
+
+
+def _ptr(a):
+    return a.ctypes.data_as(ctypes.c_void_p) if a is not None and a.size else None
+
+
+@dataclass
+class Graph:
+    """A CSR matrix A (m x n): int32 row_ptr[m+1], int32 col_idx[nnz], fp32 val[nnz]."""
+    m: int
+    n: int
+    row_ptr: np.ndarray
+    col_idx: np.ndarray
+    val: np.ndarray
+    name: str = ""
+
+    @property
+    def nnz(self) -> int:
+        return int(self.row_ptr[-1])
+
+    def digest(self) -> str:
+        h = hashlib.sha256()
+        h.update(self.row_ptr.tobytes())
+        h.update(self.col_idx.tobytes())
+        return h.hexdigest()[:16]
+
+
+def _take(h):
+    lib = _L()
+    m, n, nnz = lib.gen_rows(h), lib.gen_cols(h), lib.gen_nnz(h)
+    rp = np.zeros(m + 1, np.int32)
+    ci = np.zeros(nnz, np.int32)
+    lib.gen_copy(h, _ptr(rp), _ptr(ci))
+    lib.gen_free(h)
+    return m, n, rp, ci
+
+
+def chung_lu(n, E, alpha, dmax, seed) -> tuple:
+    return _take(_L().gen_chung_lu(n, E, alpha, dmax, seed))
+
+
+def rmat(scale, edge_factor, a, b, c, n_evil, evil_len, seed) -> tuple:
+    return _take(_L().gen_rmat(scale, edge_factor, a, b, c, n_evil, evil_len, seed))
+
+
+def random_csr(m, n, row_len, seed, canonical=True, values="int") -> Graph:
+    """CSR with the given row lengths and uniformly random columns in [0, n).
+
+    ``canonical=False`` keeps duplicate / unsorted columns (adversarial tests)."""
+    rl = np.ascontiguousarray(row_len, np.int32)
+    assert rl.shape[0] == m
+    mm, nn, rp, ci = _take(_L().gen_random_csr(m, n, _ptr(rl), int(bool(canonical)), seed))
+    g = Graph(mm, nn, rp, ci, np.zeros(ci.shape[0], np.float32), "random")
+    g.val = values_int(g.nnz, seed) if values == "int" else values_gcn(g)
+    return g
+
+
+def values_gcn(g: Graph) -> np.ndarray:
+    v = np.zeros(g.nnz, np.float32)
+    _L().gen_values_gcn(g.m, _ptr(g.row_ptr), _ptr(g.col_idx), _ptr(v))
+    return v
+
+
+def values_int(nnz, seed) -> np.ndarray:
+    v = np.zeros(nnz, np.float32)
+    _L().gen_values_int(nnz, seed, _ptr(v))
+    return v
+
+
+def dense_uniform(rows, K, seed, ld=None) -> np.ndarray:
+    ld = K if ld is None else ld
+    B = np.zeros((rows, ld), np.float32)
+    _L().gen_dense_uniform(rows, K, ld, seed, _ptr(B))
+    return B
+
+
+def dense_int(rows, K, seed, ld=None) -> np.ndarray:
+    ld = K if ld is None else ld
+    B = np.zeros((rows, ld), np.float32)
+    _L().gen_dense_int(rows, K, ld, seed, _ptr(B))
+    return B
+
+
+# --------------------------------------------------------------------------------
+# The five BASELINE.json workloads.
+#   Chung-Lu: n nodes, E undirected edges (nnz = 2E after symmetrisation), power-law
+#   weight exponent ALPHA, expected max degree dmax.  Node ids randomly permuted.
+# --------------------------------------------------------------------------------
+ALPHA = 0.75
+WORKLOADS = {
+    # name: (kind, params, seed, K list)
+    "cora": ("chung_lu", dict(n=2708, E=5278, dmax=168.0), 1, (16,)),
+    "pubmed": ("chung_lu", dict(n=19717, E=44324, dmax=171.0), 2, (16, 64)),
+    "rmat": ("rmat", dict(scale=20, edge_factor=16, a=0.57, b=0.19, c=0.19, n_evil=8,
+                          evil_len=100000), 3, (64,)),
+    "reddit": ("chung_lu", dict(n=232965, E=57307946, dmax=20000.0), 4, (64, 256)),
+    "products": ("chung_lu", dict(n=2449029, E=61859140, dmax=17000.0), 5, (128,)),
+}
+
+
+def workload(name: str, values: str = "gcn") -> Graph:
+    kind, prm, seed, _ = WORKLOADS[name]
+    if kind == "chung_lu":
+        m, n, rp, ci = chung_lu(prm["n"], prm["E"], ALPHA, prm["dmax"], seed)
+    else:
+        m, n, rp, ci = rmat(prm["scale"], prm["edge_factor"], prm["a"], prm["b"], prm["c"],
+                            prm["n_evil"], prm["evil_len"], seed)
+    g = Graph(m, n, rp, ci, np.zeros(ci.shape[0], np.float32), name)
+    g.val = values_gcn(g) if values == "gcn" else values_int(g.nnz, seed)
+    return g
+
+
+def features(name_or_rows, K, seed=None, kind="uniform") -> np.ndarray:
+    """Dense B (n x K): U[-1,1) (``uniform``) or integers in [-4, 4] (``int``)."""
+    if isinstance(name_or_rows, str):
+        rows = WORKLOADS[name_or_rows][1]["n"] if "n" in WORKLOADS[name_or_rows][1] else \
+            1 << WORKLOADS[name_or_rows][1]["scale"]
+        seed = WORKLOADS[name_or_rows][2] + 100 if seed is None else seed
+    else:
+        rows = int(name_or_rows)
+        seed = 7 if seed is None else seed
+    return dense_uniform(rows, K, seed) if kind == "uniform" else dense_int(rows, K, seed)
