@@ -1,0 +1,423 @@
+#!/usr/bin/env python
+"""MergePath-SpMM benchmark (BASELINE.json metric: SpMM GFLOP/s = 2*nnz*K / t, with the
+effective HBM GB/s and the HBM-roofline fraction beside it).
+
+One step = one pass of the whole hot path of SURVEY.md sec. 8(a) on one batch:
+a1 plan (host) + a2 partition + a4 split-row zeroing + a3 segment kernel (+ a4 carry
+reduction) and, for N > 1 GPUs, the a6 tail all-gather + tail application.  Inputs
+(A, B) are resident in HBM; L2 is flushed (a 2x-L2 write) before every timed step, and
+each step is timed with CUDA events on the launching stream.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload reddit] [--K 64]
+                    [--fixup atomic|carry] [--dtype f32|bf16] [--impl reference]
+
+N > 1: launch under torchrun (one rank per GPU, NCCL); rank 0 prints the JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import ctypes
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "SpMM GFLOP/s (2·nnz·K) & HBM GB/s vs 8 TB/s at 1/2/4/8 B200"
+FALLBACK_HBM_GBS = 6650.0   # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default="reddit")
+    ap.add_argument("--K", type=int, default=0)
+    ap.add_argument("--fixup", default="atomic")
+    ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
+    ap.add_argument("--items-per-part", type=int, default=0)
+    ap.add_argument("--min-parts", type=int, default=0)
+    ap.add_argument("--impl", default="mps", choices=["mps", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--out", default="")
+    return ap.parse_args()
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def alg_bytes(m, nnz, K, b_elt):
+    """nnz*(4 idx + 4 val) + 4*(m+1) row_ptr + b_elt*nnz*K gathered B rows
+    + 4*m*K for C."""
+    return 8 * nnz + 4 * (m + 1) + b_elt * nnz * K + 4 * m * K
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.proc, self.lines = index, None, []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.Q,
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": float(max(mx)) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_oracle_rate(g, B, K, seconds, steps=1):
+    """Time the oracle O1 (fp64, OpenMP over rows) on a bounded row sample of the same
+    workload; returns (GFLOP/s, cores, sample description, seconds per step)."""
+    import oracle as O
+    rows_all = g.m
+    deg = np.diff(g.row_ptr).astype(np.int64)
+    # calibrate on a small prefix, then size the sample to `seconds`
+    r0 = max(1, min(rows_all, 2000))
+    t = time.perf_counter()
+    O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, rows=np.arange(r0), want_bound=False)
+    dt = max(time.perf_counter() - t, 1e-6)
+    rate_nnz = deg[:r0].sum() / dt
+    want_nnz = rate_nnz * seconds / max(steps, 1)
+    cum = np.cumsum(deg)
+    R = int(np.searchsorted(cum, want_nnz)) + 1
+    R = max(1, min(rows_all, R))
+    rows = np.arange(R, dtype=np.int64)
+    times = []
+    for _ in range(steps):
+        t = time.perf_counter()
+        O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, rows=rows, want_bound=False)
+        times.append(time.perf_counter() - t)
+    nnz_s = int(cum[R - 1])
+    gflop = 2.0 * nnz_s * K / 1e9
+    tm = float(np.median(times))
+    sample = ("rows [0, %d) of %s (%d of %d nnz, %.1f%%), K=%d, fp64 oracle O1" %
+              (R, g.name, nnz_s, g.nnz, 100.0 * nnz_s / max(g.nnz, 1), K))
+    return gflop / tm, O.num_threads(), sample, tm
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle (as it stands) on a bounded sample per step."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import graphgen as G
+    g = G.workload(args.workload)
+    K = args.K or G.WORKLOADS[args.workload][3][0]
+    B = G.features(args.workload, K)
+    per_step = max(1.0, 90.0 / max(1, args.steps + args.warmup))
+    rate, cores, sample, tm = cpu_oracle_rate(g, B, K, per_step * (args.steps), args.steps)
+    line = {
+        "metric": METRIC, "value": rate, "unit": "GFLOP/s", "impl": "reference",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": tm * 1e3, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": "%s-k%d" % (args.workload, K), "n": g.m, "nnz": g.nnz, "K": K},
+        "cpu_baseline": {"value": rate, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": rate, "unit": "GFLOP/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+        "gpu_launches": 0,
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+    import graphgen as G
+    import paper_conf_ispass_shangndk23_b200 as M
+    from paper_conf_ispass_shangndk23_b200 import _lib as L
+    from paper_conf_ispass_shangndk23_b200.api import _p, _stream, FIXUP
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+
+    name = args.workload
+    K = args.K or G.WORKLOADS[name][3][0]
+    tdtype = torch.bfloat16 if args.dtype == "bf16" else torch.float32
+    b_elt = 2 if args.dtype == "bf16" else 4
+    dt_code = L.MPS_DT_BF16 if args.dtype == "bf16" else L.MPS_DT_F32
+    fix = FIXUP[args.fixup]
+
+    t0 = time.perf_counter()
+    g = G.workload(name)
+    Bh = G.features(name, K)
+    gen_s = time.perf_counter() - t0
+
+    stream = torch.cuda.current_stream(dev)
+    s_ptr = _stream(stream)
+    Bd = torch.from_numpy(Bh).to(dev).to(tdtype)
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    flush = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
+
+    launches_per_step = 0
+    seg_ms = []
+    step_ms = []
+    part_ms = []
+
+    if world == 1:
+        A = M.CSR.from_numpy(g.row_ptr, g.col_idx, g.val, g.n, device=dev)
+        a = A.struct()
+        P, Lp = M.plan(g.m, g.nnz, K, dt_code, args.items_per_part, args.min_parts)
+        cx = torch.empty(P + 1, dtype=torch.int32, device=dev)
+        cy = torch.empty(P + 1, dtype=torch.int32, device=dev)
+        C = torch.empty((g.m, K), dtype=torch.float32, device=dev)
+        nb = ctypes.c_size_t()
+        L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt_code, P, fix, ctypes.byref(nb))
+        ws = torch.empty(max(nb.value, 1), dtype=torch.uint8, device=dev)
+        tiles = -(-K // 512) if args.dtype == "f32" else -(-K // 1024)
+        launches_per_step = 1 + (1 if fix != L.MPS_FIXUP_CARRY else 0) + \
+            tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1)
+
+        def step(ev=None):
+            L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx), _p(cy),
+                            s_ptr)
+            if fix != L.MPS_FIXUP_CARRY:
+                L.mps_zero_split_rows(ctypes.byref(a), _p(cx), _p(cy), P, _p(C), K, K, s_ptr)
+            if ev is not None:
+                ev[0].record(stream)
+            L.mps_spmm_segments(ctypes.byref(a), _p(Bd), dt_code, K, K, _p(C), K, _p(cx),
+                                _p(cy), P, fix, _p(ws), nb.value, s_ptr)
+            if ev is not None:
+                ev[1].record(stream)
+        units_nnz = g.nnz
+        units_rows = g.m
+    else:
+        sh = M.ShardedSpMM(g.row_ptr, g.col_idx, g.val, g.n, K, rank, world, dev,
+                           b_dtype=tdtype, fixup=args.fixup, items_per_part=args.items_per_part,
+                           min_parts=args.min_parts)
+        P, Lp = None, None
+        tiles = -(-K // 512) if args.dtype == "f32" else -(-K // 1024)
+        launches_per_step = 2 + tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1) + 1
+
+        def step(ev=None):
+            if ev is not None:
+                ev[0].record(stream)
+            sh.local(Bd)
+            if ev is not None:
+                ev[1].record(stream)
+            tails = M.exchange_tails(sh.tail, world)
+            sh.settle(tails)
+        units_nnz = g.nnz
+        units_rows = g.m
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    # warm-up (untimed)
+    for _ in range(max(args.warmup, 0)):
+        flush.zero_()
+        step()
+    torch.cuda.synchronize(dev)
+
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+            torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(args.steps)]
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    barrier()
+    torch.cuda.synchronize(dev)
+    wall0 = time.perf_counter()
+    for i in range(args.steps):
+        flush.zero_()                     # L2 flush between timed steps (not timed)
+        evs[i][0].record(stream)
+        step((evs[i][1], evs[i][2]))
+        evs[i][3].record(stream)
+    torch.cuda.synchronize(dev)
+    barrier()
+    wall = time.perf_counter() - wall0
+    clk = clocks.stop()
+    for e in evs:
+        step_ms.append(e[0].elapsed_time(e[3]))
+        seg_ms.append(e[1].elapsed_time(e[2]))
+        part_ms.append(e[0].elapsed_time(e[1]))
+    t_step = float(np.mean(step_ms))
+    t_seg = float(np.mean(seg_ms))
+    if world > 1:
+        tt = torch.tensor([t_step, t_seg], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_step, t_seg = float(tt[0]), float(tt[1])
+
+    flops = 2.0 * units_nnz * K
+    gflops = flops / (t_step * 1e-3) / 1e9
+    bytes_alg = alg_bytes(units_rows, units_nnz, K, b_elt)
+    hbm_peak, peak_src = peaks()
+    eff_gbs = bytes_alg / (t_step * 1e-3) / 1e9
+
+    # dominant kernel roofline: the a3 segment kernel (per-rank algorithmic bytes)
+    if world == 1:
+        seg_bytes = bytes_alg
+    else:
+        y0, y1 = int(sh.Y[rank]), int(sh.Y[rank + 1])
+        seg_bytes = alg_bytes(sh.rows, y1 - y0, K, b_elt)
+    seg_gbs = seg_bytes / (t_seg * 1e-3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "traffic.json")
+    key = "%s-k%d-%s-%s" % (name, K, args.dtype, args.fixup)
+    if os.path.exists(prof) and world == 1:
+        with open(prof) as f:
+            traffic = json.load(f).get(key)
+
+    # end-to-end through the public C ABI on pinned HOST buffers (rank 0 layout, N=1)
+    e2e = None
+    if world == 1 and args.e2e_steps > 0:
+        pin = lambda x: torch.from_numpy(x).pin_memory()
+        rp_h, ci_h, va_h = pin(g.row_ptr), pin(g.col_idx), pin(g.val)
+        Bh_t = torch.from_numpy(Bh).to(tdtype).pin_memory()
+        Ch = torch.empty((g.m, K), dtype=torch.float32).pin_memory()
+        from paper_conf_ispass_shangndk23_b200.api import host_workspace_bytes
+        nbh = host_workspace_bytes(rp_h, ci_h, va_h, g.n, Bh_t, Ch, args.items_per_part,
+                                   args.min_parts, args.fixup)
+        wsh = torch.empty(nbh, dtype=torch.uint8, device=dev)
+        del A, C, ws, flush
+        torch.cuda.empty_cache()
+        ah = M.mps_csr_host(rp_h, ci_h, va_h, g.n)
+
+        def e2e_step():
+            L.mps_spmm_host(ctypes.byref(ah), _p(Bh_t), dt_code, K, K, _p(Ch), K,
+                            args.items_per_part, args.min_parts, fix, _p(wsh), nbh, s_ptr)
+        e2e_step()
+        torch.cuda.synchronize(dev)
+        e_ms = []
+        for _ in range(args.e2e_steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            e2e_step()
+            e1.record(stream)
+            torch.cuda.synchronize(dev)
+            e_ms.append(e0.elapsed_time(e1))
+        t_e2e = float(np.mean(e_ms))
+        h2d = 4 * (g.m + 1) + 8 * g.nnz + b_elt * g.n * K
+        d2h = 4 * g.m * K
+        e2e = {"value": flops / (t_e2e * 1e-3) / 1e9, "unit": "GFLOP/s",
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": t_e2e, "path": "mps_spmm_host (pinned host A, B -> C)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            rate, cores, sample, _ = cpu_oracle_rate(g, Bh if args.dtype == "f32" else
+                                                     Bd.float().cpu().numpy(), K,
+                                                     args.cpu_seconds)
+            cpu = {"value": rate, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+                   "sample": sample}
+        except Exception as e:  # pragma: no cover
+            cpu = {"value": None, "unit": "GFLOP/s", "cores": None, "kind": "oracle",
+                   "sample": "failed: %s" % e}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC,
+            "value": gflops,
+            "unit": "GFLOP/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": t_step,
+            "higher_is_better": True,
+            "scaling": "strong",
+            "vs_baseline": None,
+            "dtype": "f32" if args.dtype == "f32" else "bf16-in/f32-acc",
+            "data": "synthetic",
+            "config": {
+                "workload": "%s-k%d" % (name, K), "graph": g.name, "n": g.m, "nnz": g.nnz,
+                "K": K, "b_dtype": args.dtype, "fixup": args.fixup,
+                "num_parts": P, "items_per_part": Lp, "mode": "online (partition every step)",
+                "l2": "flushed before every timed step (2x L2 write, untimed)",
+                "parallelism": "merge-path shards x%d" % world, "graph_sha": g.digest(),
+                "gen_s": round(gen_s, 2),
+            },
+            "effective_gbs": eff_gbs,
+            "hbm_frac_step": eff_gbs / hbm_peak,
+            "partition_zero_ms": float(np.mean(part_ms)),
+            "segment_ms": t_seg,
+            "step_ms_p10_p90": [float(np.percentile(step_ms, 10)),
+                                float(np.percentile(step_ms, 90))],
+            "wall_s_timed_region": wall,
+            "roofline": {"bound": "hbm", "kernel": "segment_kernel (a3)",
+                         "achieved": seg_gbs, "peak": hbm_peak, "unit": "GB/s",
+                         "frac": seg_gbs / hbm_peak, "traffic": traffic,
+                         "algorithmic_bytes_per_launch": int(seg_bytes),
+                         "peak_source": peak_src},
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": int(launches_per_step * args.steps),
+            "clocks": clk,
+        }
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.out:
+            with open(args.out, "a") as f:
+                f.write(s + "\n")
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,187 @@
+/*
+ * mpspmm.h -- C ABI of libmpspmm.so, a B200 (sm_100a) MergePath-SpMM.
+ *
+ * Computes the GCN aggregation C = A * B (the row-wise product of PAPER.md P:41-43,
+ * sec. II) for a sparse m x n CSR matrix A and a dense, tall and thin n x K matrix B
+ * (the paper's XW), scheduled by the merge path of Alg. 1 and
+ * Alg. 2.  Citations "P:<line>" are lines of the paper text; DESIGN.md
+ * lists every reading taken where the paper is garbled or silent ("R<k>").
+ *
+ * Conventions (all entry points):
+ *  - Plain C: no C++ types, no exceptions cross this boundary.  Every function
+ *    returns an mps_status; mps_last_error() gives a thread-local detail string.
+ *  - Ownership: the caller allocates and frees every buffer (A, B, C, coordinates,
+ *    workspace, tails).  The library keeps no global state and allocates nothing
+ *    persistent; all functions are reentrant.
+ *  - Pointers are DEVICE pointers unless the parameter name ends in _host.
+ *  - Streams: every device call is asynchronous on `stream` (a cudaStream_t passed
+ *    as void*; NULL = the legacy default stream).  Only mps_validate_csr
+ *    synchronises.
+ *  - Index type: int32 row_ptr / col_idx.  M = m + nnz must be < 2^31, else
+ *    MPS_ERR_UNSUPPORTED (reading R16).
+ *  - Errors: MPS_ERR_INVALID for NULL pointers with non-zero sizes, negative sizes,
+ *    ldb < K, ldc < K, num_parts < 1, rank outside [0, world); MPS_ERR_UNSUPPORTED
+ *    for M >= 2^31 or an unknown dtype; MPS_ERR_WORKSPACE if workspace_bytes is too
+ *    small; MPS_ERR_CUDA if a launch or copy fails.  K == 0 or m == 0 is a no-op
+ *    returning MPS_OK.  Misaligned B or C selects a narrower vector path, never an
+ *    error.  CSR *content* (monotone row_ptr, columns in range) is NOT checked on the
+ *    hot path -- the method needs no preprocessing; mps_validate_csr does it.
+ */
+#ifndef MPSPMM_H
+#define MPSPMM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t mps_status;
+enum {
+    MPS_OK = 0,
+    MPS_ERR_INVALID = 1,
+    MPS_ERR_UNSUPPORTED = 2,
+    MPS_ERR_CUDA = 3,
+    MPS_ERR_WORKSPACE = 4,
+    MPS_ERR_COMM = 5
+};
+
+/* How rows split across merge-path segments are settled (a4). */
+enum {
+    MPS_FIXUP_AUTO = 0,   /* library choice (currently ATOMIC)                        */
+    MPS_FIXUP_ATOMIC = 1, /* zero split rows, then one vector red.add per partial row  */
+    MPS_FIXUP_CARRY = 2   /* partial rows to workspace, fixed-order reduction; deterministic */
+};
+
+/* Element type of B.  C is always fp32, accumulation always fp32 (reading R15). */
+enum { MPS_DT_F32 = 0, MPS_DT_BF16 = 1 };
+
+/* A: m x n CSR.  row_ptr[m+1] (row_ptr[0] = 0, row_ptr[m] = nnz), col_idx[nnz],
+ * val[nnz]; columns need not be sorted, duplicates are summed (CSR).        */
+typedef struct {
+    int64_t m, n, nnz;
+    const int32_t *row_ptr;
+    const int32_t *col_idx;
+    const float *val;
+} mps_csr;
+
+int mps_abi_version(void);
+const char *mps_status_string(mps_status s);
+const char *mps_last_error(void);
+
+/* a1 -- schedule sizing (host only, no GPU needed).  Alg. 1 lines 2-3 and
+ * sec. III-C: M = m + nnz; P = max(ceil(M / cost), min_parts);
+ * L = ceil(M / P) (reading R1).  items_per_part (the paper's merge-path cost,
+ * P:137) == 0 selects the library default for (K, b_dtype); min_parts (the paper's
+ * thread threshold) == 0 selects the library default.  Outputs P and L.    */
+mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
+                    int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out);
+
+/* a2 -- merge-path partition, Alg. 1 lines 4-7.  For p = 0..num_parts it
+ * writes the coordinate of diagonal d_p = diag_begin + min(p*L, diag_end - diag_begin)
+ * (L = items_per_part): x = max{x : x + row_ptr[x] <= d_p}, y = d_p - x
+ * (readings R4, R5).  coord_x / coord_y: caller-owned device int32[num_parts+1].
+ * Bit-exact; asynchronous on stream.                                              */
+mps_status mps_partition(const int32_t *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
+                         int64_t diag_end, int64_t num_parts, int64_t items_per_part,
+                         int32_t *coord_x, int32_t *coord_y, void *stream);
+
+/* a3+a4 -- offline SpMM with a precomputed schedule (computed once, reused).
+ * C = A * B; C is overwritten entirely (it need not be initialised: complete rows
+ * are stored, split rows are zeroed first or stored by the carry pass, empty rows
+ * get 0).  B: n rows, leading dimension ldb elements (b_dtype); C: m rows, leading
+ * dimension ldc floats.  workspace: caller-owned device memory of at least
+ * mps_spmm_workspace_bytes(...) bytes (may be NULL when that is 0).              */
+mps_status mps_spmm_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                    int64_t num_parts, int32_t fixup, size_t *bytes);
+mps_status mps_spmm(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                    float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
+                    int64_t num_parts, int32_t fixup, void *workspace, size_t workspace_bytes,
+                    void *stream);
+
+/* The two launches mps_spmm is made of, for callers that time or overlap them:
+ * mps_zero_split_rows zeroes the rows cut by a boundary of the schedule (x_p < m,
+ * y_p > row_ptr[x_p]; the atomic fix-up's precondition, reading R10);
+ * mps_spmm_segments runs a3 (+ the a4 carry reduction) and, in atomic mode,
+ * REQUIRES that mps_zero_split_rows ran earlier on the same C and schedule.       */
+mps_status mps_zero_split_rows(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
+                               int64_t num_parts, float *C, int64_t ldc, int32_t K,
+                               void *stream);
+mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                             const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                             void *workspace, size_t workspace_bytes, void *stream);
+
+/* Online convenience: a1 + a2 + a3 + a4 in one call; the partition is
+ * written into the workspace.  items_per_part / min_parts as in mps_plan.         */
+mps_status mps_spmm_online_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                           int64_t items_per_part, int64_t min_parts,
+                                           int32_t fixup, size_t *bytes);
+mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                           int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                           int64_t min_parts, int32_t fixup, void *workspace,
+                           size_t workspace_bytes, void *stream);
+
+/* End-to-end call on HOST buffers: copies A and B host->device, runs the online path
+ * and copies C device->host, all enqueued on `stream` (pinned host memory gives
+ * true async copies).  A_host holds HOST pointers.  device_workspace: caller-owned
+ * device memory of mps_spmm_host_workspace_bytes(...) bytes.  The caller
+ * synchronises the stream before reading C_host.                                 */
+mps_status mps_spmm_host_workspace_bytes(const mps_csr *A_host, int32_t K, int32_t b_dtype,
+                                         int64_t ldb, int64_t ldc, int64_t items_per_part,
+                                         int64_t min_parts, int32_t fixup, size_t *bytes);
+mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dtype,
+                         int64_t ldb, int32_t K, float *C_host, int64_t ldc,
+                         int64_t items_per_part, int64_t min_parts, int32_t fixup,
+                         void *device_workspace, size_t workspace_bytes, void *stream);
+
+/* Fig. 5 statistic: with the Alg. 2 write rules (lines 5, 9, 13 atomic,
+ * line 15 regular) for the given schedule, counts_out[0] = #atomic row updates,
+ * counts_out[1] = #regular row stores.  counts_out: device int64[2], overwritten. */
+mps_status mps_write_stats(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
+                           int64_t num_parts, int64_t *counts_out, void *stream);
+
+/* a6 -- multi-GPU merge-path sharding (north-star stage 4; not in the paper).
+ * Host closed form: shard g covers diagonals [D_g, D_{g+1}), D_g = min(g*ceil(M/G), M);
+ * (X_g, Y_g) = coordinate of D_g.  Shard g owns C rows [X_g, X_{g+1}); its tail row
+ * is X_{g+1} if that row is cut (Y_{g+1} > row_ptr[X_{g+1}]), else -1.
+ * row_ptr_host: host copy of row_ptr.  X, Y: host int32[world+1];
+ * tail_rows: host int32[world].                                                   */
+mps_status mps_shard_bounds(const int32_t *row_ptr_host, int64_t m, int64_t nnz, int32_t world,
+                            int32_t *X, int32_t *Y, int32_t *tail_rows);
+
+/* Rank-local SpMM of shard `rank`.  A->row_ptr is the GLOBAL row_ptr (device);
+ * A->col_idx / A->val point at the rank's slice, which starts at global nnz index
+ * Y[rank] (A->nnz stays the global nnz).  C_local: rows X[rank] .. X[rank+1]-1
+ * (leading dimension ldc), overwritten.  tail_out: device float[K], overwritten
+ * with the shard's partial sum of row tail_rows[rank] (zeros if there is none).
+ * X, Y, tail_rows: host arrays from mps_shard_bounds.                            */
+mps_status mps_spmm_shard_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                          const int32_t *X, int32_t rank, int32_t world,
+                                          int64_t items_per_part, int64_t min_parts,
+                                          int32_t fixup, size_t *bytes);
+mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                          int32_t K, const int32_t *X, const int32_t *Y,
+                          const int32_t *tail_rows, int32_t rank, int32_t world,
+                          int64_t items_per_part, int64_t min_parts, float *C_local,
+                          int64_t ldc, float *tail_out, int32_t fixup, void *workspace,
+                          size_t workspace_bytes, void *stream);
+
+/* After an all-gather of every rank's tail_out into tails (device float[world*K],
+ * rank-major): add the tails whose row this rank owns (owner(r) = max{g : X_g <= r})
+ * into C_local, in ascending rank order (deterministic).                         */
+mps_status mps_apply_tails(const float *tails, const int32_t *X, const int32_t *tail_rows,
+                           int32_t world, int32_t rank, int32_t K, float *C_local,
+                           int64_t ldc, void *stream);
+
+/* Debug-only validation of CSR content on the device (synchronises).  Checks
+ * row_ptr[0] == 0, row_ptr non-decreasing, row_ptr[m] == nnz, 0 <= col < n.
+ * *first_bad_host = -1 if valid, else the first offending row_ptr index (< m+1) or
+ * m + 1 + the first offending nnz index.                                          */
+mps_status mps_validate_csr(const mps_csr *A, int64_t *first_bad_host, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MPSPMM_H */

@@ -1,0 +1,15 @@
+"""B200-native MergePath-SpMM (Shan et al., ISPASS 2023): C = A * B for an ultra-sparse
+power-law CSR adjacency A and a dense, tall and thin B = X*W.
+
+The compute lives in libmpspmm.so (hand-written CUDA for sm_100a behind the C ABI of
+include/mpspmm.h).  This package is the thin Python binding: ``_lib`` mirrors the C
+entry points one to one; ``api`` and ``sharded`` marshal torch tensors to them.
+"""
+from . import _lib
+from ._lib import *  # noqa: F401,F403  (mps_* entry points, MpsError, constants)
+from .api import (CSR, Schedule, mps_csr_host, partition, plan, spmm, spmm_host,  # noqa: F401
+                  validate_csr, write_stats)
+from .sharded import ShardedSpMM, exchange_tails, shard_bounds  # noqa: F401
+
+__all__ = ["CSR", "Schedule", "plan", "partition", "spmm", "spmm_host", "write_stats",
+           "validate_csr", "ShardedSpMM", "shard_bounds", "exchange_tails"] + list(_lib.EXPORTED)

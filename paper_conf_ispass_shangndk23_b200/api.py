@@ -1,0 +1,195 @@
+"""Torch-facing helpers over the C ABI (include/mpspmm.h).
+
+PyTorch supplies device memory and the current stream; every step of the path runs in
+libmpspmm.so.  Names follow the paper: A (CSR adjacency), B (= XW),
+merge-path cost ``items_per_part``, thread floor ``min_parts``,
+offline schedule.
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+
+from . import _lib as L
+
+FIXUP = {"auto": L.MPS_FIXUP_AUTO, "atomic": L.MPS_FIXUP_ATOMIC, "carry": L.MPS_FIXUP_CARRY}
+
+
+def _p(t):
+    if t is None:
+        return None
+    if isinstance(t, np.ndarray):
+        return ctypes.c_void_p(t.ctypes.data) if t.size else None
+    return ctypes.c_void_p(t.data_ptr()) if t.numel() else None
+
+
+def _stream(stream=None):
+    s = torch.cuda.current_stream() if stream is None else stream
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _dtype_code(B):
+    if B.dtype == torch.float32:
+        return L.MPS_DT_F32
+    if B.dtype == torch.bfloat16:
+        return L.MPS_DT_BF16
+    raise TypeError("B must be float32 or bfloat16, got %s" % B.dtype)
+
+
+def _fix(f):
+    return FIXUP[f] if isinstance(f, str) else int(f)
+
+
+class CSR:
+    """A (m x n) in CSR on one device: int32 row_ptr[m+1], int32 col_idx[nnz], fp32 val."""
+
+    def __init__(self, row_ptr, col_idx, val, n_cols):
+        self.row_ptr, self.col_idx, self.val = row_ptr, col_idx, val
+        self.m = int(row_ptr.numel()) - 1
+        self.n = int(n_cols)
+        self.nnz = int(col_idx.numel())
+        assert row_ptr.dtype == torch.int32 and col_idx.dtype == torch.int32
+        assert val.dtype == torch.float32 and val.numel() == self.nnz
+
+    @classmethod
+    def from_numpy(cls, row_ptr, col_idx, val, n_cols, device="cuda"):
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(device)
+        return cls(t(row_ptr), t(col_idx), t(val), n_cols)
+
+    @property
+    def device(self):
+        return self.row_ptr.device
+
+    def struct(self) -> L.mps_csr:
+        return L.mps_csr(self.m, self.n, self.nnz, _p(self.row_ptr), _p(self.col_idx),
+                         _p(self.val))
+
+
+def mps_csr_host(row_ptr, col_idx, val, n_cols) -> L.mps_csr:
+    """An mps_csr holding HOST pointers (numpy arrays or pinned CPU tensors)."""
+    m = (row_ptr.shape[0] if isinstance(row_ptr, np.ndarray) else row_ptr.numel()) - 1
+    nnz = col_idx.shape[0] if isinstance(col_idx, np.ndarray) else col_idx.numel()
+    return L.mps_csr(m, n_cols, nnz, _p(row_ptr), _p(col_idx), _p(val))
+
+
+def plan(m, nnz, K, b_dtype=L.MPS_DT_F32, items_per_part=0, min_parts=0):
+    """a1: (P, L) = merge-path thread count and items per thread (Alg. 1 l.2-3)."""
+    P, Lp = ctypes.c_int64(), ctypes.c_int64()
+    L.mps_plan(m, nnz, K, b_dtype, items_per_part, min_parts, ctypes.byref(P), ctypes.byref(Lp))
+    return P.value, Lp.value
+
+
+def partition(A: CSR, num_parts, items_per_part, diag_begin=0, diag_end=None, stream=None):
+    """a2: coordinates (x_p, y_p), p = 0..P, of the merge-path diagonals (Alg. 1 l.4-7)."""
+    diag_end = A.m + A.nnz if diag_end is None else diag_end
+    cx = torch.empty(num_parts + 1, dtype=torch.int32, device=A.device)
+    cy = torch.empty(num_parts + 1, dtype=torch.int32, device=A.device)
+    L.mps_partition(_p(A.row_ptr), A.m, A.nnz, diag_begin, diag_end, num_parts, items_per_part,
+                    _p(cx), _p(cy), _stream(stream))
+    return cx, cy
+
+
+@dataclass
+class Schedule:
+    """An offline merge-path schedule: computed once per graph, reused."""
+    num_parts: int
+    items_per_part: int
+    coord_x: torch.Tensor
+    coord_y: torch.Tensor
+
+    @classmethod
+    def build(cls, A: CSR, K, b_dtype=torch.float32, items_per_part=0, min_parts=0, stream=None):
+        dt = L.MPS_DT_BF16 if b_dtype == torch.bfloat16 else L.MPS_DT_F32
+        P, Lp = plan(A.m, A.nnz, K, dt, items_per_part, min_parts)
+        cx, cy = partition(A, P, Lp, stream=stream)
+        return cls(P, Lp, cx, cy)
+
+
+def _ws(nbytes, device):
+    return torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=device)
+
+
+def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomic",
+         items_per_part=0, min_parts=0, out: torch.Tensor | None = None, stream=None):
+    """C = A * B (row-wise product) by MergePath-SpMM.
+
+    With ``schedule`` the offline path (mps_spmm) runs; otherwise the online path
+    (mps_spmm_online: plan + partition + SpMM).  B: (n, K) float32/bfloat16 on A's
+    device, rows may be padded (B.stride(0) = ldb >= K).  Returns C (m, K) float32."""
+    assert B.dim() == 2 and B.stride(1) == 1 and B.device == A.device
+    K = B.shape[1]
+    dt = _dtype_code(B)
+    C = torch.empty((A.m, K), dtype=torch.float32, device=A.device) if out is None else out
+    assert C.stride(1) == 1 and C.shape == (A.m, K)
+    a = A.struct()
+    nb = ctypes.c_size_t()
+    st = _stream(stream)
+    if schedule is not None:
+        L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt, schedule.num_parts, _fix(fixup),
+                                   ctypes.byref(nb))
+        ws = _ws(nb.value, A.device)
+        L.mps_spmm(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
+                   _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts, _fix(fixup),
+                   _p(ws), nb.value, st)
+    else:
+        L.mps_spmm_online_workspace_bytes(ctypes.byref(a), K, dt, items_per_part, min_parts,
+                                          _fix(fixup), ctypes.byref(nb))
+        ws = _ws(nb.value, A.device)
+        L.mps_spmm_online(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
+                          items_per_part, min_parts, _fix(fixup), _p(ws), nb.value, st)
+    return C
+
+
+def spmm_host(row_ptr, col_idx, val, n_cols, B_host, C_host=None, items_per_part=0,
+              min_parts=0, fixup="atomic", device="cuda", stream=None, workspace=None):
+    """End to end from HOST buffers (mps_spmm_host): H2D of A and B, online SpMM, D2H
+    of C, enqueued on the stream; synchronises before returning C_host."""
+    K = B_host.shape[1]
+    dt = L.MPS_DT_BF16 if B_host.dtype == torch.bfloat16 else L.MPS_DT_F32
+    m = row_ptr.numel() - 1
+    if C_host is None:
+        C_host = torch.empty((m, K), dtype=torch.float32, pin_memory=True)
+    a = mps_csr_host(row_ptr, col_idx, val, n_cols)
+    nb = ctypes.c_size_t()
+    L.mps_spmm_host_workspace_bytes(ctypes.byref(a), K, dt, B_host.stride(0), C_host.stride(0),
+                                    items_per_part, min_parts, _fix(fixup), ctypes.byref(nb))
+    ws = workspace if workspace is not None and workspace.numel() >= nb.value else \
+        _ws(nb.value, device)
+    s = torch.cuda.current_stream() if stream is None else stream
+    L.mps_spmm_host(ctypes.byref(a), _p(B_host), dt, B_host.stride(0), K, _p(C_host),
+                    C_host.stride(0), items_per_part, min_parts, _fix(fixup), _p(ws),
+                    ws.numel(), _stream(s))
+    s.synchronize()
+    return C_host
+
+
+def host_workspace_bytes(row_ptr, col_idx, val, n_cols, B_host, C_host, items_per_part=0,
+                         min_parts=0, fixup="atomic"):
+    K = B_host.shape[1]
+    dt = L.MPS_DT_BF16 if B_host.dtype == torch.bfloat16 else L.MPS_DT_F32
+    a = mps_csr_host(row_ptr, col_idx, val, n_cols)
+    nb = ctypes.c_size_t()
+    L.mps_spmm_host_workspace_bytes(ctypes.byref(a), K, dt, B_host.stride(0), C_host.stride(0),
+                                    items_per_part, min_parts, _fix(fixup), ctypes.byref(nb))
+    return nb.value
+
+
+def write_stats(A: CSR, schedule: Schedule, stream=None):
+    """Fig. 5 statistic: (#atomic row updates, #regular row stores) under Alg. 2."""
+    cnt = torch.empty(2, dtype=torch.int64, device=A.device)
+    a = A.struct()
+    L.mps_write_stats(ctypes.byref(a), _p(schedule.coord_x), _p(schedule.coord_y),
+                      schedule.num_parts, _p(cnt), _stream(stream))
+    c = cnt.cpu()
+    return int(c[0]), int(c[1])
+
+
+def validate_csr(A: CSR, stream=None) -> int:
+    """-1 if A's CSR content is valid, else the first offending index (synchronises)."""
+    a = A.struct()
+    bad = ctypes.c_int64()
+    L.mps_validate_csr(ctypes.byref(a), ctypes.byref(bad), _stream(stream))
+    return bad.value

@@ -1,0 +1,603 @@
+// capi.cu -- the extern "C" boundary of libmpspmm.so (include/mpspmm.h): argument
+// validation, schedule sizing (a1), workspace layout, column tiling and launch order.
+#include <cstdio>
+#include <cstring>
+#include <cstdarg>
+#include <vector>
+
+#include "mps_internal.cuh"
+
+namespace {
+
+thread_local char g_err[512] = "";
+
+mps_status fail(mps_status st, const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return st;
+}
+
+mps_status cuda_fail(cudaError_t e, const char *where) {
+    return fail(MPS_ERR_CUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+#define MPS_CUDA(call, where)                                   \
+    do {                                                        \
+        cudaError_t e__ = (call);                               \
+        if (e__ != cudaSuccess) return cuda_fail(e__, where);   \
+    } while (0)
+
+constexpr int64_t kMaxIndex = (int64_t)1 << 31;
+constexpr int64_t kDefaultMinParts = 8 * 148;  // ~ the paper's 1024-thread floor
+
+inline size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+inline int elt_bytes(int32_t dt) { return dt == MPS_DT_BF16 ? 2 : 4; }
+
+// Default merge-path cost (items per warp segment) by feature width; the paper tunes
+// this per K (Fig. 6); these are B200 values.
+int64_t default_cost(int32_t K, int32_t dt) {
+    (void)dt;
+    if (K <= 32) return 256;
+    if (K <= 128) return 512;
+    return 256;
+}
+
+struct Vec {
+    int W = 1;     // elements per lane access
+    int tile = 0;  // columns per launch (multiple of 32*W)
+};
+
+// Widest lane vector the alignment of B and C allows, preferring widths that fill the
+// 32 lanes of the warp; V = ceil(K_tile / (32 W)) <= 4 slots per lane.
+Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C, int64_t ldc) {
+    const int eb = elt_bytes(dt);
+    const int cand_f32[3] = {4, 2, 1};
+    const int cand_bf[4] = {8, 4, 2, 1};
+    const int *cand = dt == MPS_DT_BF16 ? cand_bf : cand_f32;
+    const int nc = dt == MPS_DT_BF16 ? 4 : 3;
+    auto ok = [&](int W) {
+        const int cw = W < 4 ? W : 4;  // C is written in float(W<=4) or float4 pieces
+        return K % W == 0 && ldb % W == 0 && ((uintptr_t)B % (size_t)(W * eb)) == 0 &&
+               ldc % cw == 0 && ((uintptr_t)C % (size_t)(cw * 4)) == 0;
+    };
+    Vec v;
+    for (int i = 0; i < nc && v.tile == 0; ++i)
+        if (ok(cand[i]) && K >= 32 * cand[i]) { v.W = cand[i]; v.tile = 32 * cand[i] * 4; }
+    for (int i = 0; i < nc && v.tile == 0; ++i)
+        if (ok(cand[i])) { v.W = cand[i]; v.tile = 32 * cand[i] * 4; }
+    if (v.tile == 0) { v.W = 1; v.tile = 128; }
+    return v;
+}
+
+mps_status check_csr(const mps_csr *A, bool device_ptrs_needed = true) {
+    if (!A) return fail(MPS_ERR_INVALID, "A is NULL");
+    if (A->m < 0 || A->n < 0 || A->nnz < 0) return fail(MPS_ERR_INVALID, "negative CSR size");
+    if (A->m + A->nnz >= kMaxIndex || A->n >= kMaxIndex)
+        return fail(MPS_ERR_UNSUPPORTED, "m + nnz = %lld >= 2^31 (int32 indices)",
+                    (long long)(A->m + A->nnz));
+    if (device_ptrs_needed && A->m > 0 && !A->row_ptr) return fail(MPS_ERR_INVALID, "row_ptr NULL");
+    if (device_ptrs_needed && A->nnz > 0 && (!A->col_idx || !A->val))
+        return fail(MPS_ERR_INVALID, "col_idx/val NULL");
+    return MPS_OK;
+}
+
+mps_status check_dense(const void *B, int32_t dt, int64_t ldb, int32_t K, const float *C,
+                       int64_t ldc, const mps_csr *A) {
+    if (dt != MPS_DT_F32 && dt != MPS_DT_BF16) return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", dt);
+    if (K < 0) return fail(MPS_ERR_INVALID, "K < 0");
+    if (K > 0 && (ldb < K || ldc < K)) return fail(MPS_ERR_INVALID, "ldb/ldc < K");
+    if (K > 0 && A->m > 0 && !C) return fail(MPS_ERR_INVALID, "C NULL");
+    if (K > 0 && A->nnz > 0 && !B) return fail(MPS_ERR_INVALID, "B NULL");
+    return MPS_OK;
+}
+
+int64_t carry_kpad(int32_t K, const Vec &v) {
+    const int64_t kt = K < v.tile ? K : v.tile;
+    return (int64_t)align_up((size_t)kt, 8);
+}
+
+size_t carry_bytes(int64_t P, int32_t K, const Vec &v) {
+    return (size_t)P * 2 * (size_t)carry_kpad(K, v) * sizeof(float);
+}
+
+int resolve_fix(int32_t fixup) { return fixup == MPS_FIXUP_CARRY ? mps::FIX_CARRY : mps::FIX_ATOMIC; }
+
+// host coordinate of diagonal d (shard bounds): x = max{x : x + rp[x] <= d}
+int64_t host_diag_x(const int32_t *rp, int64_t m, int64_t nnz, int64_t d) {
+    int64_t lo = (d > nnz ? d - nnz : 0) + 1, hi = (d < m ? d : m) + 1;
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        if (mid + (int64_t)rp[mid] > d) hi = mid;
+        else lo = mid + 1;
+    }
+    return lo - 1;
+}
+
+// Run a3 (+ a4 carry reduction) over all column tiles for a ready schedule.
+mps_status run_segments(mps::SegArgs base, int32_t dt, int32_t K, const Vec &v, int fix,
+                        void *workspace, cudaStream_t s) {
+    const int eb = elt_bytes(dt);
+    for (int32_t c0 = 0; c0 < K; c0 += v.tile) {
+        mps::SegArgs a = base;
+        const int32_t kt = (K - c0) < v.tile ? (K - c0) : v.tile;
+        a.K = kt;
+        a.B = (const char *)base.B + (size_t)c0 * eb;
+        a.C = base.C ? base.C + c0 : nullptr;
+        a.tail = base.tail ? base.tail + c0 : nullptr;
+        a.rec = (float *)workspace;
+        a.kpad = (int32_t)carry_kpad(K, v);
+        // TMA staging needs col and val equally aligned modulo 16 B
+        a.direct = ((((uintptr_t)base.col) ^ ((uintptr_t)base.val)) & 15u) != 0;
+        const int V = (kt + 32 * v.W - 1) / (32 * v.W);
+        MPS_CUDA(mps::launch_segments(a, dt, v.W, V, fix, s), "segment kernel");
+        if (fix == mps::FIX_CARRY) MPS_CUDA(mps::launch_carry_reduce(a, s), "carry reduce");
+    }
+    return MPS_OK;
+}
+
+}  // namespace
+
+namespace mps {
+int num_sms() {
+    static int cache[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148;
+    if (cache[dev] == 0) {
+        int v = 0;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0)
+            v = 148;
+        cache[dev] = v;
+    }
+    return cache[dev];
+}
+}  // namespace mps
+
+extern "C" {
+
+int mps_abi_version(void) { return 1; }
+
+const char *mps_status_string(mps_status s) {
+    switch (s) {
+    case MPS_OK: return "MPS_OK";
+    case MPS_ERR_INVALID: return "MPS_ERR_INVALID";
+    case MPS_ERR_UNSUPPORTED: return "MPS_ERR_UNSUPPORTED";
+    case MPS_ERR_CUDA: return "MPS_ERR_CUDA";
+    case MPS_ERR_WORKSPACE: return "MPS_ERR_WORKSPACE";
+    case MPS_ERR_COMM: return "MPS_ERR_COMM";
+    default: return "MPS_ERR_UNKNOWN";
+    }
+}
+
+const char *mps_last_error(void) { return g_err; }
+
+mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
+                    int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out) {
+    if (m < 0 || nnz < 0 || K < 0 || items_per_part < 0 || min_parts < 0)
+        return fail(MPS_ERR_INVALID, "negative plan argument");
+    if (!num_parts_out || !items_per_part_out) return fail(MPS_ERR_INVALID, "NULL output");
+    if (b_dtype != MPS_DT_F32 && b_dtype != MPS_DT_BF16)
+        return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", b_dtype);
+    if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    const int64_t cost = items_per_part ? items_per_part : default_cost(K, b_dtype);
+    const int64_t pmin = min_parts ? min_parts : kDefaultMinParts;
+    const int64_t M = m + nnz;                      // Alg. 1 line 2
+    int64_t P = (M + cost - 1) / cost;              // threads = merge_items / cost
+    if (P < pmin) P = pmin;                         // thread floor
+    *num_parts_out = P;
+    *items_per_part_out = (M + P - 1) / P;          // Alg. 1 line 3 (reading R1)
+    return MPS_OK;
+}
+
+mps_status mps_partition(const int32_t *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
+                         int64_t diag_end, int64_t num_parts, int64_t items_per_part,
+                         int32_t *coord_x, int32_t *coord_y, void *stream) {
+    if (m < 0 || nnz < 0 || num_parts < 1 || items_per_part < 0)
+        return fail(MPS_ERR_INVALID, "bad partition sizes");
+    if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (diag_begin < 0 || diag_end < diag_begin || diag_end > m + nnz)
+        return fail(MPS_ERR_INVALID, "diagonal range outside [0, m + nnz]");
+    if (!row_ptr || !coord_x || !coord_y) return fail(MPS_ERR_INVALID, "NULL pointer");
+    MPS_CUDA(mps::launch_partition(row_ptr, m, nnz, diag_begin, diag_end - diag_begin, num_parts,
+                                   items_per_part, coord_x, coord_y, nullptr, 0, 0, 0, -1,
+                                   nullptr, (cudaStream_t)stream),
+             "partition kernel");
+    return MPS_OK;
+}
+
+mps_status mps_spmm_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                    int64_t num_parts, int32_t fixup, size_t *bytes) {
+    mps_status st = check_csr(A, false);
+    if (st) return st;
+    if (!bytes || num_parts < 1 || K < 0) return fail(MPS_ERR_INVALID, "bad arguments");
+    if (b_dtype != MPS_DT_F32 && b_dtype != MPS_DT_BF16)
+        return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", b_dtype);
+    // worst case over alignments: the narrowest vector gives the smallest tile
+    Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
+    Vec vmin;
+    vmin.W = 1;
+    vmin.tile = 128;
+    size_t need = resolve_fix(fixup) == mps::FIX_CARRY
+                      ? (carry_bytes(num_parts, K, v) > carry_bytes(num_parts, K, vmin)
+                             ? carry_bytes(num_parts, K, v) : carry_bytes(num_parts, K, vmin))
+                      : 0;
+    *bytes = need;
+    return MPS_OK;
+}
+
+mps_status mps_zero_split_rows(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
+                               int64_t num_parts, float *C, int64_t ldc, int32_t K,
+                               void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (num_parts < 1 || K < 0 || (K > 0 && ldc < K)) return fail(MPS_ERR_INVALID, "bad arguments");
+    if (K == 0 || A->m == 0) return MPS_OK;
+    if (!coord_x || !coord_y || !C) return fail(MPS_ERR_INVALID, "NULL pointer");
+    MPS_CUDA(mps::launch_zero_split(A->row_ptr, (int32_t)A->m, coord_x, coord_y, num_parts, C,
+                                    ldc, 0, K, -1, nullptr, (cudaStream_t)stream),
+             "zero split rows");
+    return MPS_OK;
+}
+
+mps_status mps_spmm(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                    float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
+                    int64_t num_parts, int32_t fixup, void *workspace, size_t workspace_bytes,
+                    void *stream) {
+    if (resolve_fix(fixup) == mps::FIX_ATOMIC) {
+        mps_status st = check_csr(A);
+        if (st) return st;
+        if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
+        if (num_parts < 1) return fail(MPS_ERR_INVALID, "num_parts < 1");
+        if (K == 0 || A->m == 0) return MPS_OK;
+        if ((st = mps_zero_split_rows(A, coord_x, coord_y, num_parts, C, ldc, K, stream)))
+            return st;
+    }
+    return mps_spmm_segments(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                             workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                             const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                             void *workspace, size_t workspace_bytes, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
+    if (num_parts < 1) return fail(MPS_ERR_INVALID, "num_parts < 1");
+    if (K == 0 || A->m == 0) return MPS_OK;
+    if (!coord_x || !coord_y) return fail(MPS_ERR_INVALID, "NULL coordinates");
+    const int fix = resolve_fix(fixup);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc);
+    if (fix == mps::FIX_CARRY && workspace_bytes < carry_bytes(num_parts, K, v))
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes,
+                    carry_bytes(num_parts, K, v));
+    if (fix == mps::FIX_CARRY && !workspace) return fail(MPS_ERR_WORKSPACE, "workspace NULL");
+    cudaStream_t s = (cudaStream_t)stream;
+    mps::SegArgs a{};
+    a.rp = A->row_ptr;
+    a.col = A->col_idx;
+    a.val = A->val;
+    a.B = B;
+    a.ldb = ldb;
+    a.C = C;
+    a.ldc = ldc;
+    a.row_base = 0;
+    a.m = (int32_t)A->m;
+    a.cx = coord_x;
+    a.cy = coord_y;
+    a.P = num_parts;
+    a.tail_row = -1;
+    a.tail = nullptr;
+    a.nnz_end = A->nnz;
+    return run_segments(a, b_dtype, K, v, fix, workspace, s);
+}
+
+static size_t online_bytes(int64_t P, int32_t K, const Vec &v, int fix) {
+    size_t b = align_up((size_t)(P + 1) * 4, 256) * 2;
+    if (fix == mps::FIX_CARRY) b += carry_bytes(P, K, v);
+    return b;
+}
+
+mps_status mps_spmm_online_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                           int64_t items_per_part, int64_t min_parts,
+                                           int32_t fixup, size_t *bytes) {
+    mps_status st = check_csr(A, false);
+    if (st) return st;
+    if (!bytes) return fail(MPS_ERR_INVALID, "bytes NULL");
+    int64_t P, L;
+    if ((st = mps_plan(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
+    Vec vmin;
+    vmin.W = 1;
+    vmin.tile = 128;
+    const Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
+    const int fix = resolve_fix(fixup);
+    size_t a = online_bytes(P, K, v, fix), b = online_bytes(P, K, vmin, fix);
+    *bytes = a > b ? a : b;
+    return MPS_OK;
+}
+
+mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                           int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                           int64_t min_parts, int32_t fixup, void *workspace,
+                           size_t workspace_bytes, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
+    if (K == 0 || A->m == 0) return MPS_OK;
+    int64_t P, L;
+    if ((st = mps_plan(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
+    const int fix = resolve_fix(fixup);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc);
+    const size_t need = online_bytes(P, K, v, fix);
+    if (!workspace || workspace_bytes < need)
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
+    cudaStream_t s = (cudaStream_t)stream;
+    int32_t *cx = (int32_t *)workspace;
+    int32_t *cy = (int32_t *)((char *)workspace + align_up((size_t)(P + 1) * 4, 256));
+    void *rec = (char *)workspace + align_up((size_t)(P + 1) * 4, 256) * 2;
+    MPS_CUDA(mps::launch_partition(A->row_ptr, A->m, A->nnz, 0, A->m + A->nnz, P, L, cx, cy,
+                                   fix == mps::FIX_ATOMIC ? C : nullptr, ldc, 0, K, -1, nullptr,
+                                   s),
+             "partition kernel");
+    mps::SegArgs a{};
+    a.rp = A->row_ptr;
+    a.col = A->col_idx;
+    a.val = A->val;
+    a.B = B;
+    a.ldb = ldb;
+    a.C = C;
+    a.ldc = ldc;
+    a.row_base = 0;
+    a.m = (int32_t)A->m;
+    a.cx = cx;
+    a.cy = cy;
+    a.P = P;
+    a.tail_row = -1;
+    a.tail = nullptr;
+    a.nnz_end = A->nnz;
+    return run_segments(a, b_dtype, K, v, fix, rec, s);
+}
+
+// ----------------------------------------------------------------------------------
+// host-buffer end-to-end call
+// ----------------------------------------------------------------------------------
+struct HostLayout {
+    size_t rp, ci, val, B, C, ws, total;
+};
+
+static HostLayout host_layout(const mps_csr *A, int32_t dt, int64_t ldb, int64_t ldc,
+                              size_t online) {
+    HostLayout h;
+    size_t o = 0;
+    h.rp = o; o += align_up((size_t)(A->m + 1) * 4, 256);
+    h.ci = o; o += align_up((size_t)A->nnz * 4, 256);
+    h.val = o; o += align_up((size_t)A->nnz * 4, 256);
+    h.B = o; o += align_up((size_t)A->n * (size_t)ldb * elt_bytes(dt), 256);
+    h.C = o; o += align_up((size_t)A->m * (size_t)ldc * 4, 256);
+    h.ws = o; o += online;
+    h.total = o;
+    return h;
+}
+
+mps_status mps_spmm_host_workspace_bytes(const mps_csr *A_host, int32_t K, int32_t b_dtype,
+                                         int64_t ldb, int64_t ldc, int64_t items_per_part,
+                                         int64_t min_parts, int32_t fixup, size_t *bytes) {
+    size_t online = 0;
+    mps_status st = mps_spmm_online_workspace_bytes(A_host, K, b_dtype, items_per_part,
+                                                    min_parts, fixup, &online);
+    if (st) return st;
+    *bytes = host_layout(A_host, b_dtype, ldb, ldc, online).total;
+    return MPS_OK;
+}
+
+mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dtype,
+                         int64_t ldb, int32_t K, float *C_host, int64_t ldc,
+                         int64_t items_per_part, int64_t min_parts, int32_t fixup,
+                         void *device_workspace, size_t workspace_bytes, void *stream) {
+    mps_status st = check_csr(A_host);
+    if (st) return st;
+    if ((st = check_dense(B_host, b_dtype, ldb, K, C_host, ldc, A_host))) return st;
+    if (K == 0 || A_host->m == 0) return MPS_OK;
+    size_t online = 0;
+    if ((st = mps_spmm_online_workspace_bytes(A_host, K, b_dtype, items_per_part, min_parts,
+                                              fixup, &online)))
+        return st;
+    const HostLayout h = host_layout(A_host, b_dtype, ldb, ldc, online);
+    if (!device_workspace || workspace_bytes < h.total)
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, h.total);
+    cudaStream_t s = (cudaStream_t)stream;
+    char *w = (char *)device_workspace;
+    const size_t bbytes = (size_t)A_host->n * (size_t)ldb * elt_bytes(b_dtype);
+    MPS_CUDA(cudaMemcpyAsync(w + h.rp, A_host->row_ptr, (size_t)(A_host->m + 1) * 4,
+                             cudaMemcpyHostToDevice, s), "H2D row_ptr");
+    if (A_host->nnz) {
+        MPS_CUDA(cudaMemcpyAsync(w + h.ci, A_host->col_idx, (size_t)A_host->nnz * 4,
+                                 cudaMemcpyHostToDevice, s), "H2D col_idx");
+        MPS_CUDA(cudaMemcpyAsync(w + h.val, A_host->val, (size_t)A_host->nnz * 4,
+                                 cudaMemcpyHostToDevice, s), "H2D val");
+    }
+    if (bbytes) MPS_CUDA(cudaMemcpyAsync(w + h.B, B_host, bbytes, cudaMemcpyHostToDevice, s), "H2D B");
+    mps_csr Ad = *A_host;
+    Ad.row_ptr = (const int32_t *)(w + h.rp);
+    Ad.col_idx = (const int32_t *)(w + h.ci);
+    Ad.val = (const float *)(w + h.val);
+    if ((st = mps_spmm_online(&Ad, w + h.B, b_dtype, ldb, K, (float *)(w + h.C), ldc,
+                              items_per_part, min_parts, fixup, w + h.ws, online, stream)))
+        return st;
+    MPS_CUDA(cudaMemcpyAsync(C_host, w + h.C, (size_t)A_host->m * (size_t)ldc * 4,
+                             cudaMemcpyDeviceToHost, s), "D2H C");
+    return MPS_OK;
+}
+
+mps_status mps_write_stats(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
+                           int64_t num_parts, int64_t *counts_out, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (num_parts < 1 || !coord_x || !coord_y || !counts_out)
+        return fail(MPS_ERR_INVALID, "bad arguments");
+    MPS_CUDA(mps::launch_write_stats(A->row_ptr, (int32_t)A->m, coord_x, coord_y, num_parts,
+                                     counts_out, (cudaStream_t)stream),
+             "write stats");
+    return MPS_OK;
+}
+
+// ----------------------------------------------------------------------------------
+// sharding (a6)
+// ----------------------------------------------------------------------------------
+mps_status mps_shard_bounds(const int32_t *row_ptr_host, int64_t m, int64_t nnz, int32_t world,
+                            int32_t *X, int32_t *Y, int32_t *tail_rows) {
+    if (m < 0 || nnz < 0 || world < 1) return fail(MPS_ERR_INVALID, "bad shard arguments");
+    if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (!row_ptr_host || !X || !Y || !tail_rows) return fail(MPS_ERR_INVALID, "NULL pointer");
+    const int64_t M = m + nnz;
+    const int64_t per = (M + world - 1) / world;
+    for (int32_t g = 0; g <= world; ++g) {
+        int64_t d = (int64_t)g * per;
+        if (d > M) d = M;
+        const int64_t x = host_diag_x(row_ptr_host, m, nnz, d);
+        X[g] = (int32_t)x;
+        Y[g] = (int32_t)(d - x);
+    }
+    for (int32_t g = 0; g < world; ++g) {
+        const int32_t r = X[g + 1];
+        tail_rows[g] = (r < m && Y[g + 1] > row_ptr_host[r]) ? r : -1;
+    }
+    return MPS_OK;
+}
+
+static mps_status shard_plan(const int32_t *X, const int32_t *Y, int32_t rank, int32_t K,
+                             int32_t dt, int64_t ipp, int64_t minp, int64_t *P, int64_t *L,
+                             int64_t *D0, int64_t *span) {
+    *D0 = (int64_t)X[rank] + Y[rank];
+    const int64_t D1 = (int64_t)X[rank + 1] + Y[rank + 1];
+    *span = D1 - *D0;
+    if (*span < 0) return fail(MPS_ERR_INVALID, "shard bounds not monotone");
+    // local plan over the shard's merge items (items of rows counted as rows here)
+    return mps_plan(*span, 0, K, dt, ipp, minp, P, L);
+}
+
+mps_status mps_spmm_shard_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                          const int32_t *X, int32_t rank, int32_t world,
+                                          int64_t items_per_part, int64_t min_parts,
+                                          int32_t fixup, size_t *bytes) {
+    mps_status st = check_csr(A, false);
+    if (st) return st;
+    if (!X || !bytes || world < 1 || rank < 0 || rank >= world)
+        return fail(MPS_ERR_INVALID, "bad shard arguments");
+    (void)X;
+    // Y is not needed for the size: the span is at most ceil(M/world)
+    const int64_t M = A->m + A->nnz;
+    const int64_t span = (M + world - 1) / world;
+    int64_t P, L;
+    if ((st = mps_plan(span, 0, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
+    Vec vmin;
+    vmin.W = 1;
+    vmin.tile = 128;
+    const Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
+    const int fix = resolve_fix(fixup);
+    size_t a = online_bytes(P, K, v, fix), b = online_bytes(P, K, vmin, fix);
+    *bytes = a > b ? a : b;
+    return MPS_OK;
+}
+
+mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                          int32_t K, const int32_t *X, const int32_t *Y,
+                          const int32_t *tail_rows, int32_t rank, int32_t world,
+                          int64_t items_per_part, int64_t min_parts, float *C_local,
+                          int64_t ldc, float *tail_out, int32_t fixup, void *workspace,
+                          size_t workspace_bytes, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (!X || !Y || !tail_rows || world < 1 || rank < 0 || rank >= world)
+        return fail(MPS_ERR_INVALID, "bad shard arguments");
+    if ((st = check_dense(B, b_dtype, ldb, K, C_local ? C_local : (float *)B, ldc, A))) return st;
+    if (K == 0) return MPS_OK;
+    if (!tail_out) return fail(MPS_ERR_INVALID, "tail_out NULL");
+    cudaStream_t s = (cudaStream_t)stream;
+    MPS_CUDA(cudaMemsetAsync(tail_out, 0, (size_t)K * 4, s), "zero tail");
+    int64_t P, L, D0, span;
+    if ((st = shard_plan(X, Y, rank, K, b_dtype, items_per_part, min_parts, &P, &L, &D0, &span)))
+        return st;
+    if (span == 0) return MPS_OK;
+    const int fix = resolve_fix(fixup);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C_local ? C_local : tail_out, ldc);
+    const size_t need = online_bytes(P, K, v, fix);
+    if (!workspace || workspace_bytes < need)
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
+    int32_t *cx = (int32_t *)workspace;
+    int32_t *cy = (int32_t *)((char *)workspace + align_up((size_t)(P + 1) * 4, 256));
+    void *rec = (char *)workspace + align_up((size_t)(P + 1) * 4, 256) * 2;
+    const int32_t trow = tail_rows[rank];
+    MPS_CUDA(mps::launch_partition(A->row_ptr, A->m, A->nnz, D0, span, P, L, cx, cy,
+                                   fix == mps::FIX_ATOMIC ? C_local : nullptr, ldc, X[rank], K,
+                                   trow, fix == mps::FIX_ATOMIC ? tail_out : nullptr, s),
+             "partition kernel");
+    mps::SegArgs a{};
+    a.rp = A->row_ptr;
+    // col/val hold global nnz [Y[rank], ...): shift so that col[j] is global nnz j
+    a.col = (const int32_t *)((uintptr_t)A->col_idx - (uintptr_t)Y[rank] * 4);
+    a.val = (const float *)((uintptr_t)A->val - (uintptr_t)Y[rank] * 4);
+    a.B = B;
+    a.ldb = ldb;
+    a.C = C_local;
+    a.ldc = ldc;
+    a.row_base = X[rank];
+    a.m = (int32_t)A->m;
+    a.cx = cx;
+    a.cy = cy;
+    a.P = P;
+    a.tail_row = trow;
+    a.tail = tail_out;
+    a.nnz_end = Y[rank + 1];
+    return run_segments(a, b_dtype, K, v, fix, rec, s);
+}
+
+mps_status mps_apply_tails(const float *tails, const int32_t *X, const int32_t *tail_rows,
+                           int32_t world, int32_t rank, int32_t K, float *C_local,
+                           int64_t ldc, void *stream) {
+    if (!X || !tail_rows || world < 1 || rank < 0 || rank >= world || K < 0 || ldc < K)
+        return fail(MPS_ERR_INVALID, "bad apply_tails arguments");
+    std::vector<int32_t> mine;
+    int32_t row = -1;
+    for (int32_t h = 0; h < world; ++h) {
+        const int32_t r = tail_rows[h];
+        if (r < 0) continue;
+        int32_t owner = 0;
+        for (int32_t g = 0; g < world; ++g)
+            if (X[g] <= r) owner = g;
+        if (owner != rank) continue;
+        mine.push_back(h);
+        row = r;
+    }
+    if (mine.empty() || K == 0) return MPS_OK;
+    if (!tails || !C_local) return fail(MPS_ERR_INVALID, "NULL pointer");
+    MPS_CUDA(mps::launch_apply_tails(tails, K, mine.data(), (int32_t)mine.size(),
+                                     C_local + (int64_t)(row - X[rank]) * ldc,
+                                     (cudaStream_t)stream),
+             "apply tails");
+    return MPS_OK;
+}
+
+mps_status mps_validate_csr(const mps_csr *A, int64_t *first_bad_host, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (!first_bad_host) return fail(MPS_ERR_INVALID, "first_bad_host NULL");
+    *first_bad_host = -1;
+    if (A->m == 0 && A->nnz == 0) return MPS_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    unsigned long long *d = nullptr;
+    MPS_CUDA(cudaMallocAsync((void **)&d, sizeof(*d), s), "alloc");
+    const unsigned long long init = ~0ull;
+    MPS_CUDA(cudaMemcpyAsync(d, &init, sizeof(init), cudaMemcpyHostToDevice, s), "H2D");
+    MPS_CUDA(mps::launch_validate(A->row_ptr, A->col_idx, A->m, A->n, A->nnz, d, s), "validate");
+    unsigned long long h = 0;
+    MPS_CUDA(cudaMemcpyAsync(&h, d, sizeof(h), cudaMemcpyDeviceToHost, s), "D2H");
+    MPS_CUDA(cudaFreeAsync(d, s), "free");
+    MPS_CUDA(cudaStreamSynchronize(s), "sync");
+    *first_bad_host = (h == ~0ull) ? -1 : (int64_t)h;
+    return MPS_OK;
+}
+
+}  // extern "C"

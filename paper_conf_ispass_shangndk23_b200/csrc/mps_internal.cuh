@@ -1,0 +1,268 @@
+// mps_internal.cuh -- device helpers and kernel interfaces of libmpspmm (sm_100a).
+//
+// Product code.  Shares nothing with oracle/ (the CPU checker): no headers, tables or
+// helpers.  Paper citations "P:<line>" refer to PAPER.md (MergePath-SpMM, ISPASS'23).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <stdint.h>
+
+#include "../../include/mpspmm.h"
+
+namespace mps {
+
+constexpr int kBlock = 256;  // threads per CTA for every kernel of the library
+
+enum Fix : int { FIX_ATOMIC = 1, FIX_CARRY = 2 };
+
+// Per-launch arguments of the segment kernel (a3 + a4).  Indices are global merge-path
+// coordinates; col/val are pre-offset so that col[j] is global nnz j (shards hold a
+// slice); C row r lives at C + (r - row_base) * ldc; the row `tail_row` (a shard's cut
+// last row) is redirected to `tail`.
+struct SegArgs {
+    const int32_t *rp;
+    const int32_t *col;
+    const float *val;
+    const void *B;
+    int64_t ldb;
+    int32_t K;          // columns of this column tile
+    float *C;
+    int64_t ldc;
+    int64_t row_base;
+    int32_t m;          // rows of the global A
+    const int32_t *cx;
+    const int32_t *cy;
+    int64_t P;
+    int32_t tail_row;   // -1: none
+    float *tail;
+    float *rec;         // carry records [P][2][kpad]
+    int32_t kpad;
+    int64_t nnz_end;    // one past the last readable (global) nnz index of col/val
+    int32_t direct;     // 1: col/val misaligned relative to each other -> no TMA staging
+};
+
+// Host launchers (defined in the .cu files).
+cudaError_t launch_partition(const int32_t *rp, int64_t m, int64_t nnz, int64_t d0,
+                             int64_t span, int64_t P, int64_t L, int32_t *cx, int32_t *cy,
+                             float *zero_C, int64_t ldc, int64_t row_base, int32_t K,
+                             int32_t tail_row, float *tail, cudaStream_t s);
+cudaError_t launch_zero_split(const int32_t *rp, int32_t m, const int32_t *cx,
+                              const int32_t *cy, int64_t P, float *C, int64_t ldc,
+                              int64_t row_base, int32_t K, int32_t tail_row, float *tail,
+                              cudaStream_t s);
+cudaError_t launch_segments(const SegArgs &a, int b_dtype, int W, int V, int fix,
+                            cudaStream_t s);
+cudaError_t launch_carry_reduce(const SegArgs &a, cudaStream_t s);
+cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx, int32_t n,
+                               float *row, cudaStream_t s);
+cudaError_t launch_write_stats(const int32_t *rp, int32_t m, const int32_t *cx,
+                               const int32_t *cy, int64_t P, int64_t *counts, cudaStream_t s);
+cudaError_t launch_validate(const int32_t *rp, const int32_t *col, int64_t m, int64_t n,
+                            int64_t nnz, unsigned long long *first_bad, cudaStream_t s);
+
+int num_sms();
+
+// ---------------------------------------------------------------------------------
+// device helpers
+// ---------------------------------------------------------------------------------
+__device__ __forceinline__ int ld_stream_i32(const int32_t *p) {
+    int v;
+    asm volatile("ld.global.cs.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ float ld_stream_f32(const float *p) {
+    float v;
+    asm volatile("ld.global.cs.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}
+
+// L2 cache policies: B rows are re-gathered (keep them: evict_last); col/val and C are
+// streamed once (evict_first).
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+// W consecutive elements of B (type TB) as one raw vector gather (read-only path, no L1
+// allocation, L2 evict_last), converted to fp32 at use.
+template <typename TB, int W> struct BVec;
+
+template <> struct BVec<float, 4> {
+    using raw = float4;
+    static __device__ __forceinline__ raw load(const float *p, uint64_t pol) {
+        raw r;
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p), "l"(pol));
+        return r;
+    }
+    static __device__ __forceinline__ void cvt(const raw &r, float (&o)[4]) {
+        o[0] = r.x; o[1] = r.y; o[2] = r.z; o[3] = r.w;
+    }
+};
+template <> struct BVec<float, 2> {
+    using raw = float2;
+    static __device__ __forceinline__ raw load(const float *p, uint64_t pol) {
+        raw r;
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f32 {%0,%1}, [%2], %3;"
+                     : "=f"(r.x), "=f"(r.y) : "l"(p), "l"(pol));
+        return r;
+    }
+    static __device__ __forceinline__ void cvt(const raw &r, float (&o)[2]) {
+        o[0] = r.x; o[1] = r.y;
+    }
+};
+template <> struct BVec<float, 1> {
+    using raw = float;
+    static __device__ __forceinline__ raw load(const float *p, uint64_t pol) {
+        raw r;
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;"
+                     : "=f"(r) : "l"(p), "l"(pol));
+        return r;
+    }
+    static __device__ __forceinline__ void cvt(const raw &r, float (&o)[1]) { o[0] = r; }
+};
+
+__device__ __forceinline__ float bf_lo(uint32_t w) { return __uint_as_float(w << 16); }
+__device__ __forceinline__ float bf_hi(uint32_t w) { return __uint_as_float(w & 0xffff0000u); }
+
+template <> struct BVec<__nv_bfloat16, 8> {
+    using raw = uint4;
+    static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
+        raw r;
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.b32 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+        return r;
+    }
+    static __device__ __forceinline__ void cvt(const raw &r, float (&o)[8]) {
+        o[0] = bf_lo(r.x); o[1] = bf_hi(r.x); o[2] = bf_lo(r.y); o[3] = bf_hi(r.y);
+        o[4] = bf_lo(r.z); o[5] = bf_hi(r.z); o[6] = bf_lo(r.w); o[7] = bf_hi(r.w);
+    }
+};
+template <> struct BVec<__nv_bfloat16, 4> {
+    using raw = uint2;
+    static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
+        raw r;
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.b32 {%0,%1}, [%2], %3;"
+                     : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
+        return r;
+    }
+    static __device__ __forceinline__ void cvt(const raw &r, float (&o)[4]) {
+        o[0] = bf_lo(r.x); o[1] = bf_hi(r.x); o[2] = bf_lo(r.y); o[3] = bf_hi(r.y);
+    }
+};
+template <> struct BVec<__nv_bfloat16, 2> {
+    using raw = uint32_t;
+    static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
+        raw r;
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;"
+                     : "=r"(r) : "l"(p), "l"(pol));
+        return r;
+    }
+    static __device__ __forceinline__ void cvt(const raw &r, float (&o)[2]) {
+        o[0] = bf_lo(r); o[1] = bf_hi(r);
+    }
+};
+template <> struct BVec<__nv_bfloat16, 1> {
+    using raw = unsigned short;
+    static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
+        raw r;
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b16 %0, [%1], %2;"
+                     : "=h"(r) : "l"(p), "l"(pol));
+        return r;
+    }
+    static __device__ __forceinline__ void cvt(const raw &r, float (&o)[1]) {
+        o[0] = __uint_as_float((uint32_t)r << 16);
+    }
+};
+
+// base + idx * stride as ONE mad.wide.u32 (IMAD.WIDE.U32 with a 64-bit addend).
+__device__ __forceinline__ const char *row_addr(const char *base, uint32_t idx, uint32_t stride) {
+    uint64_t r;
+    asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(idx), "r"(stride), "l"(base));
+    return reinterpret_cast<const char *>(r);
+}
+
+// acc[0..1] += s * b[0..1] as one packed FFMA2 (sm_100: fma.rn.f32x2).
+__device__ __forceinline__ void fma2(float &a0, float &a1, float s, float b0, float b1) {
+    asm("{\n\t.reg .b64 acc, bb, ss;\n\t"
+        "mov.b64 acc, {%0, %1};\n\tmov.b64 bb, {%3, %4};\n\tmov.b64 ss, {%2, %2};\n\t"
+        "fma.rn.f32x2 acc, ss, bb, acc;\n\tmov.b64 {%0, %1}, acc;\n\t}"
+        : "+f"(a0), "+f"(a1) : "f"(s), "f"(b0), "f"(b1));
+}
+
+// ---- mbarrier + 1-D TMA bulk copy (cp.async.bulk) -----------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_fence_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"
+                 :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred P;\n\t"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+        "@!P bra WAIT_%=;\n\t}"
+        :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// global -> shared bulk copy of `bytes` (multiple of 16, both addresses 16-B aligned),
+// completion counted on `bar`; L2 evict_first (streamed once).
+__device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t bytes,
+                                            uint64_t *bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1], %2, [%3], %4;"
+        :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
+}
+
+// W consecutive fp32 of C: streaming store, or vector reduction (red.global.add.v4.f32).
+template <int W> struct CVec;
+template <> struct CVec<1> {
+    static __device__ __forceinline__ void store(float *p, const float (&v)[1]) { __stcs(p, v[0]); }
+    static __device__ __forceinline__ void add(float *p, const float (&v)[1]) { atomicAdd(p, v[0]); }
+};
+template <> struct CVec<2> {
+    static __device__ __forceinline__ void store(float *p, const float (&v)[2]) {
+        __stcs(reinterpret_cast<float2 *>(p), make_float2(v[0], v[1]));
+    }
+    static __device__ __forceinline__ void add(float *p, const float (&v)[2]) {
+        atomicAdd(reinterpret_cast<float2 *>(p), make_float2(v[0], v[1]));
+    }
+};
+template <> struct CVec<4> {
+    static __device__ __forceinline__ void store(float *p, const float (&v)[4]) {
+        __stcs(reinterpret_cast<float4 *>(p), make_float4(v[0], v[1], v[2], v[3]));
+    }
+    static __device__ __forceinline__ void add(float *p, const float (&v)[4]) {
+        atomicAdd(reinterpret_cast<float4 *>(p), make_float4(v[0], v[1], v[2], v[3]));
+    }
+};
+template <> struct CVec<8> {
+    static __device__ __forceinline__ void store(float *p, const float (&v)[8]) {
+        __stcs(reinterpret_cast<float4 *>(p), make_float4(v[0], v[1], v[2], v[3]));
+        __stcs(reinterpret_cast<float4 *>(p + 4), make_float4(v[4], v[5], v[6], v[7]));
+    }
+    static __device__ __forceinline__ void add(float *p, const float (&v)[8]) {
+        atomicAdd(reinterpret_cast<float4 *>(p), make_float4(v[0], v[1], v[2], v[3]));
+        atomicAdd(reinterpret_cast<float4 *>(p + 4), make_float4(v[4], v[5], v[6], v[7]));
+    }
+};
+
+}  // namespace mps

@@ -1,0 +1,95 @@
+"""a6: merge-path sharding of C = A*B over G GPUs (north-star stage 4; not in the paper).
+
+One process per GPU (torch.distributed, NCCL over NVLink/NVSwitch).  The merge path of
+A is cut into G equal slices of rows + non-zeros (the paper's Alg. 1 applied with G
+"threads"), so every GPU gets the same item count and, by the byte balance of
+DESIGN.md, the same memory traffic.  B is replicated (read-only); GPU g owns C rows
+[X_g, X_{g+1}).  The only exchange is the tail record of a row cut by a slice edge:
+one all-gather of G x K floats, after which each owner adds the tails of its row in
+ascending rank order (deterministic).
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+from . import _lib as L
+from .api import CSR, _p, _stream, _fix, _dtype_code, _ws
+
+
+def shard_bounds(row_ptr_host: np.ndarray, world: int):
+    """Host closed form (mps_shard_bounds): X, Y (int32[world+1]) and tail rows."""
+    rp = np.ascontiguousarray(row_ptr_host, np.int32)
+    m, nnz = rp.shape[0] - 1, int(rp[-1])
+    X = np.zeros(world + 1, np.int32)
+    Y = np.zeros(world + 1, np.int32)
+    T = np.zeros(world, np.int32)
+    L.mps_shard_bounds(_p(rp), m, nnz, world, _p(X), _p(Y), _p(T))
+    return X, Y, T
+
+
+def exchange_tails(tail: torch.Tensor, world: int, group=None) -> torch.Tensor:
+    """All-gather every rank's tail vector (K floats) -> (world*K,) rank-major.
+
+    This is the path's only collective (NCCL on GPUs, gloo in the CPU tests)."""
+    out = torch.empty(world * tail.numel(), dtype=tail.dtype, device=tail.device)
+    if world == 1:
+        out.copy_(tail.reshape(-1))
+        return out
+    dist.all_gather_into_tensor(out, tail.reshape(-1).contiguous(), group=group)
+    return out
+
+
+class ShardedSpMM:
+    """Rank-local state of a merge-path sharded SpMM.
+
+    row_ptr/col_idx/val: the global CSR on the host (numpy); every rank computes the
+    same bounds, uploads the full row_ptr and only its own [Y_g, Y_{g+1}) slice."""
+
+    def __init__(self, row_ptr, col_idx, val, n_cols, K, rank, world, device,
+                 b_dtype=torch.float32, fixup="atomic", items_per_part=0, min_parts=0,
+                 group=None):
+        self.rank, self.world, self.group, self.K = rank, world, group, K
+        self.device = torch.device(device)
+        self.fixup, self.ipp, self.minp = fixup, items_per_part, min_parts
+        self.X, self.Y, self.T = shard_bounds(row_ptr, world)
+        y0, y1 = int(self.Y[rank]), int(self.Y[rank + 1])
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(self.device)
+        self.row_ptr = t(row_ptr)
+        self.col = t(col_idx[y0:y1])
+        self.val = t(val[y0:y1])
+        self.m, self.n, self.nnz = len(row_ptr) - 1, int(n_cols), int(row_ptr[-1])
+        self.row0 = int(self.X[rank])
+        self.rows = int(self.X[rank + 1]) - self.row0
+        self.C = torch.empty((max(self.rows, 1), K), dtype=torch.float32, device=self.device)
+        self.tail = torch.zeros(K, dtype=torch.float32, device=self.device)
+        self.a = L.mps_csr(self.m, self.n, self.nnz, _p(self.row_ptr), _p(self.col), _p(self.val))
+        dt = L.MPS_DT_BF16 if b_dtype == torch.bfloat16 else L.MPS_DT_F32
+        nb = ctypes.c_size_t()
+        L.mps_spmm_shard_workspace_bytes(ctypes.byref(self.a), K, dt, _p(self.X), rank, world,
+                                         items_per_part, min_parts, _fix(fixup), ctypes.byref(nb))
+        self.ws = _ws(nb.value, self.device)
+
+    def local(self, B: torch.Tensor, stream=None):
+        """a2-a4 on this rank's slice: C rows [X_g, X_{g+1}) and the tail vector."""
+        dt = _dtype_code(B)
+        L.mps_spmm_shard(ctypes.byref(self.a), _p(B), dt, B.stride(0), self.K, _p(self.X),
+                         _p(self.Y), _p(self.T), self.rank, self.world, self.ipp, self.minp,
+                         _p(self.C) if self.rows > 0 else None, self.C.stride(0), _p(self.tail),
+                         _fix(self.fixup), _p(self.ws), self.ws.numel(), _stream(stream))
+        return self.C[: self.rows], self.tail
+
+    def settle(self, tails_all: torch.Tensor, stream=None):
+        """Add the gathered tails owned by this rank (ascending rank order)."""
+        L.mps_apply_tails(_p(tails_all), _p(self.X), _p(self.T), self.world, self.rank, self.K,
+                          _p(self.C) if self.rows > 0 else None, self.C.stride(0),
+                          _stream(stream))
+        return self.C[: self.rows]
+
+    def __call__(self, B: torch.Tensor):
+        self.local(B)
+        tails = exchange_tails(self.tail, self.world, self.group)
+        return self.settle(tails)

@@ -1,0 +1,79 @@
+"""The C-ABI library loads on a GPU-less host and exports every symbol that
+include/mpspmm.h declares; host-only entry points (plan, shard bounds) agree with the
+oracle and report errors through status codes.  No device compute here."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import graphgen as G
+import oracle as O
+import paper_conf_ispass_shangndk23_b200 as M
+from paper_conf_ispass_shangndk23_b200 import _lib
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_functions():
+    with open(os.path.join(ROOT, "include", "mpspmm.h")) as f:
+        src = f.read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(mps_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_header_symbols_exported():
+    names = declared_functions()
+    assert len(names) >= 17
+    lib = ctypes.CDLL(_lib.LIB_PATH)
+    for n in names:
+        assert hasattr(lib, n), n
+        assert n in _lib.EXPORTED, n     # and bound one-to-one in Python
+    assert set(_lib.EXPORTED) == set(names)
+
+
+def test_abi_version_and_status_strings():
+    assert M.mps_abi_version() == 1
+    assert M.mps_status_string(0) == b"MPS_OK"
+    assert M.mps_status_string(4) == b"MPS_ERR_WORKSPACE"
+
+
+def test_plan_matches_oracle():
+    rs = np.random.RandomState(0)
+    for _ in range(500):
+        m, nnz = int(rs.randint(0, 10 ** 7)), int(rs.randint(0, 10 ** 8))
+        cost, pmin = int(rs.randint(1, 5000)), int(rs.randint(1, 20000))
+        assert M.plan(m, nnz, 64, 0, cost, pmin) == O.plan(m, nnz, cost, pmin)
+    P, L = M.plan(232965, 114615892, 64)          # library defaults
+    assert P * L >= 232965 + 114615892
+
+
+def test_plan_errors():
+    P, L = ctypes.c_int64(), ctypes.c_int64()
+    with pytest.raises(M.MpsError) as e:
+        M.mps_plan(1, 1, 8, 9, 0, 0, ctypes.byref(P), ctypes.byref(L))
+    assert e.value.status == M.MPS_ERR_UNSUPPORTED
+    with pytest.raises(M.MpsError) as e:
+        M.mps_plan(2 ** 31, 0, 8, 0, 0, 0, ctypes.byref(P), ctypes.byref(L))
+    assert e.value.status == M.MPS_ERR_UNSUPPORTED
+    with pytest.raises(M.MpsError) as e:
+        M.mps_plan(-1, 0, 8, 0, 0, 0, ctypes.byref(P), ctypes.byref(L))
+    assert e.value.status == M.MPS_ERR_INVALID
+    with pytest.raises(M.MpsError) as e:
+        M.mps_spmm_online(None, None, 0, 8, 8, None, 8, 0, 0, 1, None, 0, None)
+    assert e.value.status == M.MPS_ERR_INVALID
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8, 64])
+def test_shard_bounds_match_oracle(world):
+    for name in ("cora", "pubmed"):
+        g = G.workload(name)
+        X, Y, T = M.shard_bounds(g.row_ptr, world)
+        ox, oy, ot = O.shard(g.row_ptr, world)
+        assert np.array_equal(X, ox) and np.array_equal(Y, oy) and np.array_equal(T, ot)
+    rl = np.zeros(9, np.int32)
+    rl[4] = 1000
+    g = G.random_csr(9, 9, rl, 1)
+    X, Y, T = M.shard_bounds(g.row_ptr, world)
+    assert np.array_equal(T, O.shard(g.row_ptr, world)[2])

@@ -1,0 +1,324 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bars: merge-path coordinates bit-exact; integer-valued inputs
+bit-exact in every fix-up mode, schedule and shard count; float inputs within the
+north-star tolerance |C - C_ref| <= 1e-5 (|A||B|) + 1e-7 (oracle.check, O8).
+"""
+import numpy as np
+import pytest
+import torch
+
+import graphgen as G
+import oracle as O
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_ispass_shangndk23_b200 as M
+    from paper_conf_ispass_shangndk23_b200 import api
+
+
+def dev(g):
+    return M.CSR.from_numpy(g.row_ptr, g.col_idx, g.val, g.n)
+
+
+def tB(B, dtype=torch.float32):
+    return torch.from_numpy(B).to("cuda").to(dtype)
+
+
+def rand_graph(rs, m, n, max_len, seed, dup=False, vals="int"):
+    kind = rs.randint(4)
+    if kind == 0:
+        rl = rs.randint(0, max_len + 1, size=m)
+    elif kind == 1:
+        rl = np.where(rs.rand(m) < 0.6, 0, rs.randint(0, max_len + 1, size=m))
+    elif kind == 2:
+        rl = rs.randint(0, 3, size=m)
+        if m:
+            rl[rs.randint(m)] = max_len * 20
+    else:
+        rl = rs.randint(0, max_len + 1, size=m)
+        if m:
+            rl[0] = max_len * 10
+            rl[-1] = max_len * 10
+    return G.random_csr(m, n, rl.astype(np.int32), seed, canonical=not dup, values=vals)
+
+
+# --------------------------------------------------------------------------------
+# a2: partition, bit-exact
+# --------------------------------------------------------------------------------
+@pytest.mark.parametrize("name", ["cora", "pubmed"])
+@pytest.mark.parametrize("cost", [1, 7, 64, 512, 100000])
+def test_partition_bit_exact_workloads(name, cost):
+    g = G.workload(name)
+    A = dev(g)
+    P, L = M.plan(g.m, g.nnz, 16, 0, cost, 1)
+    assert (P, L) == O.plan(g.m, g.nnz, cost, 1)
+    cx, cy = M.partition(A, P, L)
+    ox, oy = O.partition(g.row_ptr, P, L)
+    assert np.array_equal(cx.cpu().numpy(), ox) and np.array_equal(cy.cpu().numpy(), oy)
+
+
+def test_partition_bit_exact_random_and_subranges():
+    rs = np.random.RandomState(0)
+    for trial in range(60):
+        g = rand_graph(rs, int(rs.randint(0, 300)), 50, 9, seed=trial)
+        A = dev(g)
+        M_ = g.m + g.nnz
+        b = int(rs.randint(0, M_ + 1))
+        e = int(rs.randint(b, M_ + 1))
+        P = int(rs.randint(1, 70))
+        L = int(rs.randint(0, 2 * max(1, (e - b) // P) + 2))
+        cx, cy = M.partition(A, P, L, b, e)
+        ox, oy = O.partition(g.row_ptr, P, L, b, e)
+        assert np.array_equal(cx.cpu().numpy(), ox) and np.array_equal(cy.cpu().numpy(), oy)
+
+
+def test_partition_fig3():
+    rp = np.array([0, 8, 12, 13, 14, 15, 15, 16, 16, 16, 16], np.int32)
+    g = G.random_csr(10, 10, np.diff(rp).astype(np.int32), 1)
+    cx, cy = M.partition(dev(g), 4, 7)
+    assert cx.cpu().tolist() == [0, 0, 2, 6, 10] and cy.cpu().tolist()[:3] == [0, 7, 12]
+
+
+# --------------------------------------------------------------------------------
+# a3 + a4: SpMM, integer inputs bit-exact
+# --------------------------------------------------------------------------------
+KS = [1, 3, 4, 15, 16, 17, 32, 64, 100, 128, 256, 257, 520]
+
+
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+@pytest.mark.parametrize("K", KS)
+def test_spmm_integer_exact_random(fixup, K):
+    rs = np.random.RandomState(K)
+    for trial in range(6):
+        g = rand_graph(rs, int(rs.randint(1, 400)), 300, 12, seed=trial, dup=bool(trial % 2))
+        B = G.dense_int(300, K, seed=trial)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        A = dev(g)
+        for cost in (1, 5, 33, 256, 10 ** 6):
+            sch = M.Schedule.build(A, K, items_per_part=cost, min_parts=1)
+            C = torch.full((g.m, K), float("nan"), device="cuda")
+            M.spmm(A, tB(B), schedule=sch, fixup=fixup, out=C)
+            assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (trial, cost)
+            C2 = M.spmm(A, tB(B), fixup=fixup, items_per_part=cost, min_parts=1)
+            assert np.array_equal(C2.cpu().numpy().astype(np.float64), ref), (trial, cost)
+
+
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_spmm_padded_and_misaligned(fixup):
+    rs = np.random.RandomState(3)
+    g = rand_graph(rs, 500, 200, 10, seed=3)
+    A = dev(g)
+    for K, ld, off in [(64, 72, 0), (64, 68, 1), (30, 33, 0), (128, 130, 2), (16, 20, 3)]:
+        Bfull = G.dense_int(200, ld, seed=K)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, np.ascontiguousarray(Bfull[:, off:off + K]),
+                             want_bound=False)
+        Bt = tB(Bfull)[:, off:off + K]          # row stride ld, base offset by `off` floats
+        Cbig = torch.full((g.m, K + 5), float("nan"), device="cuda")
+        C = Cbig[:, 1:1 + K]                    # ldc = K + 5, misaligned base
+        M.spmm(A, Bt, fixup=fixup, out=C, items_per_part=37, min_parts=1)
+        assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (K, ld, off)
+        assert torch.isnan(Cbig[:, 0]).all() and torch.isnan(Cbig[:, K + 1:]).all()
+
+
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_spmm_degenerate(fixup):
+    K = 8
+    cases = []
+    cases.append(G.random_csr(0, 5, np.zeros(0, np.int32), 1))            # m = 0
+    cases.append(G.random_csr(7, 5, np.zeros(7, np.int32), 1))            # nnz = 0
+    for pos in (0, 3, 6):                                                 # one row holds all
+        rl = np.zeros(7, np.int32)
+        rl[pos] = 3000
+        cases.append(G.random_csr(7, 50, rl, pos))
+    for L in (9, 10, 11):                                                 # rows L-1, L, L+1
+        rl = np.full(40, L - 1, np.int32)
+        cases.append(G.random_csr(40, 50, rl, L))
+    for g in cases:
+        B = G.dense_int(g.n, K, seed=2)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        A = dev(g)
+        for cost, pmin in [(1, 1), (10, 1), (10 ** 6, 1), (4, 10 ** 4)]:   # L = 1, P > M
+            C = torch.full((g.m, K), float("nan"), device="cuda")
+            M.spmm(A, tB(B), fixup=fixup, out=C, items_per_part=cost, min_parts=pmin)
+            assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
+
+
+def test_identity_and_ones():
+    n, K = 3001, 64
+    rp = np.arange(n + 1, dtype=np.int32)
+    A = M.CSR.from_numpy(rp, np.arange(n, dtype=np.int32), np.ones(n, np.float32), n)
+    B = G.dense_uniform(n, K, seed=5)
+    C = M.spmm(A, tB(B))
+    assert torch.equal(C.cpu(), torch.from_numpy(B))
+    g = G.workload("pubmed")
+    C1 = M.spmm(dev(g), torch.ones(g.n, 16, device="cuda")).cpu().numpy()
+    rows = np.repeat(np.arange(g.m), np.diff(g.row_ptr))
+    wdeg = np.bincount(rows, weights=g.val.astype(np.float64), minlength=g.m)
+    assert np.all(C1 == C1[:, :1])
+    np.testing.assert_allclose(C1[:, 0], wdeg, rtol=1e-5, atol=1e-7)
+
+
+# --------------------------------------------------------------------------------
+# float inputs within the north-star tolerance
+# --------------------------------------------------------------------------------
+@pytest.mark.parametrize("name,K", [("cora", 16), ("pubmed", 16), ("pubmed", 64)])
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_spmm_tolerance_workloads(name, K, fixup):
+    g = G.workload(name)
+    B = G.features(name, K)
+    ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B)
+    A = dev(g)
+    for cost in (0, 8, 64):
+        C = torch.full((g.m, K), float("nan"), device="cuda")
+        M.spmm(A, tB(B), fixup=fixup, out=C, items_per_part=cost)
+        r = O.check(C.cpu().numpy(), ref, bnd)
+        assert r["ok"], r
+
+
+def test_carry_is_deterministic():
+    g = G.workload("pubmed")
+    B = tB(G.features("pubmed", 64))
+    A = dev(g)
+    a = M.spmm(A, B, fixup="carry", items_per_part=16)
+    b = M.spmm(A, B, fixup="carry", items_per_part=16)
+    assert torch.equal(a, b)
+
+
+def test_bf16_B_within_tolerance():
+    g = G.workload("pubmed")
+    for K in (16, 64, 128, 256, 24):
+        B = G.features("pubmed", K)
+        Bb = torch.from_numpy(B).to(torch.bfloat16)
+        Bq = Bb.to(torch.float32).numpy()              # the oracle sees the rounded B
+        ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bq)
+        for fixup in ("atomic", "carry"):
+            C = M.spmm(dev(g), Bb.cuda(), fixup=fixup, items_per_part=50)
+            r = O.check(C.cpu().numpy(), ref, bnd)
+            assert r["ok"], (K, fixup, r)
+
+
+# --------------------------------------------------------------------------------
+# Fig. 5 statistic, validation, host end-to-end
+# --------------------------------------------------------------------------------
+def test_write_stats_match_alg2_counters():
+    rs = np.random.RandomState(8)
+    for trial in range(20):
+        g = rand_graph(rs, int(rs.randint(1, 300)), 40, 9, seed=trial)
+        A = dev(g)
+        for cost in (1, 6, 50):
+            sch = M.Schedule.build(A, 4, items_per_part=cost, min_parts=1)
+            B = G.dense_int(40, 2, seed=1)
+            _, na, nr = O.alg2_emulate(g.row_ptr, g.col_idx, g.val, B,
+                                       sch.coord_x.cpu().numpy(), sch.coord_y.cpu().numpy())
+            assert M.write_stats(A, sch) == (na, nr)
+
+
+def test_validate_csr():
+    g = G.workload("cora")
+    assert M.validate_csr(dev(g)) == -1
+    bad = g.col_idx.copy()
+    bad[100] = g.n + 5
+    assert M.validate_csr(M.CSR.from_numpy(g.row_ptr, bad, g.val, g.n)) == g.m + 1 + 100
+
+
+def test_spmm_host_end_to_end():
+    g = G.workload("pubmed")
+    B = G.features("pubmed", 64)
+    ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B)
+    pin = lambda a: torch.from_numpy(a).pin_memory()
+    C = M.spmm_host(pin(g.row_ptr), pin(g.col_idx), pin(g.val), g.n, pin(B))
+    assert O.check(C.numpy(), ref, bnd)["ok"]
+
+
+# --------------------------------------------------------------------------------
+# a6: sharding, loopback on one GPU (every rank run in turn, tails gathered by copy)
+# --------------------------------------------------------------------------------
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_sharded_loopback_exact(fixup):
+    rs = np.random.RandomState(12)
+    graphs = [rand_graph(rs, 300, 100, 10, seed=s) for s in range(4)]
+    rl = np.ones(50, np.int32)
+    rl[20] = 5000                                       # one row spanning 3+ shards
+    graphs.append(G.random_csr(50, 100, rl, 9))
+    graphs.append(G.workload("cora", values="int"))
+    for g in graphs:
+        K = 24
+        B = G.dense_int(g.n, K, seed=4)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for world in (1, 2, 3, 4, 8):
+            shards = [M.ShardedSpMM(g.row_ptr, g.col_idx, g.val, g.n, K, r, world, "cuda",
+                                    fixup=fixup, items_per_part=7, min_parts=1)
+                      for r in range(world)]
+            X, Y, T = shards[0].X, shards[0].Y, shards[0].T
+            ox, oy, ot = O.shard(g.row_ptr, world)
+            assert np.array_equal(X, ox) and np.array_equal(Y, oy) and np.array_equal(T, ot)
+            Bt = tB(B)
+            for s in shards:
+                s.local(Bt)
+            tails = torch.cat([s.tail for s in shards])
+            out = np.zeros_like(ref)
+            for r, s in enumerate(shards):
+                # local result before the exchange equals the oracle's shard_local
+                Cl, tail = O.shard_local(g.row_ptr, g.col_idx, g.val, B, X, Y, r)
+                assert np.array_equal(s.tail.cpu().numpy().astype(np.float64), tail)
+                Cr = s.settle(tails).cpu().numpy().astype(np.float64)
+                out[X[r]:X[r + 1]] = Cr
+            assert np.array_equal(out, ref), (world, fixup)
+
+
+# --------------------------------------------------------------------------------
+# full-size BASELINE workloads: sampled rows + whole-matrix properties
+# --------------------------------------------------------------------------------
+def _sampled_check(g, K, fixup, cost=0, dtype=torch.float32, seed=0):
+    B = G.features(g.name, K)
+    Bt = tB(B, dtype)
+    if dtype == torch.bfloat16:
+        B = Bt.float().cpu().numpy()
+    A = dev(g)
+    sch = M.Schedule.build(A, K, b_dtype=dtype, items_per_part=cost)
+    C = torch.full((g.m, K), float("nan"), device="cuda")
+    M.spmm(A, Bt, schedule=sch, fixup=fixup, out=C)
+    torch.cuda.synchronize()
+    assert not torch.isnan(C).any()
+    cx = sch.coord_x.cpu().numpy()
+    cy = sch.coord_y.cpu().numpy()
+    split = cx[(cx < g.m) & (cy > g.row_ptr[np.minimum(cx, g.m)])]
+    deg = np.diff(g.row_ptr)
+    rs = np.random.RandomState(seed)
+    rows = np.unique(np.concatenate([
+        rs.choice(g.m, 3000), split[rs.choice(len(split), min(len(split), 2000))] if len(split) else [],
+        np.argsort(deg)[-50:], [0, g.m - 1]]).astype(np.int64))
+    ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, rows=rows)
+    r = O.check(C[torch.from_numpy(rows).cuda()].cpu().numpy(), ref, bnd)
+    assert r["ok"], r
+    # whole matrix: sum_i C[i,:] = w^T B with w[c] = sum of A's column c (fp64, any size)
+    w = np.bincount(g.col_idx, weights=g.val.astype(np.float64), minlength=g.n)
+    colsum_ref = w @ B.astype(np.float64)
+    colsum_abs = np.abs(w) @ np.abs(B.astype(np.float64))
+    colsum = C.double().sum(0).cpu().numpy()
+    assert np.all(np.abs(colsum - colsum_ref) <= 1e-5 * colsum_abs + 1e-3)
+    return sch
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_rmat_full_size(fixup):
+    g = G.workload("rmat")
+    _sampled_check(g, 64, fixup)
+
+
+@pytest.mark.slow
+def test_reddit_full_size_k64_and_k256():
+    g = G.workload("reddit")
+    _sampled_check(g, 64, "atomic")
+    _sampled_check(g, 256, "atomic")
+    _sampled_check(g, 64, "carry")
+
+
+@pytest.mark.slow
+def test_products_full_size_k128():
+    g = G.workload("products")
+    _sampled_check(g, 128, "atomic")
+    _sampled_check(g, 128, "atomic", dtype=torch.bfloat16)
