@@ -49,6 +49,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--out", default="")
+    ap.add_argument("--flush", default="write", choices=["write", "read", "none"],
+                    help="L2 flush before each timed step: write (default) or read a 2x-L2 "
+                         "buffer, or none")
     return ap.parse_args()
 
 
@@ -213,6 +216,13 @@ def main():
     Bd = torch.from_numpy(Bh).to(dev).to(tdtype)
     l2 = torch.cuda.get_device_properties(dev).L2_cache_size
     flush = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
+    flush_sink = torch.empty(1, dtype=torch.float32, device=dev)
+
+    def do_flush():
+        if args.flush == "write":
+            flush.zero_()
+        elif args.flush == "read":
+            torch.sum(flush, dim=0, out=flush_sink[0])
 
     launches_per_step = 0
     seg_ms = []
@@ -271,7 +281,7 @@ def main():
 
     # warm-up (untimed)
     for _ in range(max(args.warmup, 0)):
-        flush.zero_()
+        do_flush()
         step()
     torch.cuda.synchronize(dev)
 
@@ -285,7 +295,7 @@ def main():
     torch.cuda.synchronize(dev)
     wall0 = time.perf_counter()
     for i in range(args.steps):
-        flush.zero_()                     # L2 flush between timed steps (not timed)
+        do_flush()                        # L2 flush between timed steps (not timed)
         evs[i][0].record(stream)
         step((evs[i][1], evs[i][2]))
         evs[i][3].record(stream)
@@ -389,7 +399,9 @@ def main():
                 "workload": "%s-k%d" % (name, K), "graph": g.name, "n": g.m, "nnz": g.nnz,
                 "K": K, "b_dtype": args.dtype, "fixup": args.fixup,
                 "num_parts": P, "items_per_part": Lp, "mode": "online (partition every step)",
-                "l2": "flushed before every timed step (2x L2 write, untimed)",
+                "l2": {"write": "flushed before every timed step (2x L2 write, untimed)",
+                       "read": "flushed before every timed step (2x L2 read, untimed)",
+                       "none": "not flushed (col/val > L2)"}[args.flush],
                 "parallelism": "merge-path shards x%d" % world, "graph_sha": g.digest(),
                 "gen_s": round(gen_s, 2),
             },
@@ -397,6 +409,7 @@ def main():
             "hbm_frac_step": eff_gbs / hbm_peak,
             "partition_zero_ms": float(np.mean(part_ms)),
             "segment_ms": t_seg,
+            "segment_ms_steps": [round(x, 4) for x in seg_ms],
             "step_ms_p10_p90": [float(np.percentile(step_ms, 10)),
                                 float(np.percentile(step_ms, 90))],
             "wall_s_timed_region": wall,

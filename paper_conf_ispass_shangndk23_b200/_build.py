@@ -38,14 +38,17 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(d) <= t for d in _deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date():
+def build(force: bool = False, verbose: bool = False, lib: str = None, defines=()) -> str:
+    """Build libmpspmm.so (or, for experiments, `lib` with extra -D `defines`)."""
+    target = lib or LIB
+    if not force and lib is None and up_to_date():
         return LIB
-    os.makedirs(OBJ, exist_ok=True)
-    flags = [f for f in FLAGS if f != "--use_fast_math=false"]
+    obj_dir = OBJ if lib is None else OBJ + "_" + os.path.basename(lib).replace(".so", "")
+    os.makedirs(obj_dir, exist_ok=True)
+    flags = [f for f in FLAGS if f != "--use_fast_math=false"] + ["-D" + d for d in defines]
 
     def compile_one(src):
-        obj = os.path.join(OBJ, os.path.basename(src) + ".o")
+        obj = os.path.join(obj_dir, os.path.basename(src) + ".o")
         cmd = [NVCC, *ARCH, *flags, "-I", os.path.join(ROOT, "include"), "-c", src, "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
@@ -56,16 +59,22 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
         objs = list(ex.map(compile_one, _sources()))
-    tmp = LIB + ".tmp%d" % os.getpid()
+    tmp = target + ".tmp%d" % os.getpid()
     cmd = [NVCC, *ARCH, "-shared", "-Xcompiler", "-fPIC", *objs, "-o", tmp]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("nvcc link failed:\n%s\n%s" % (r.stdout, r.stderr))
-    os.replace(tmp, LIB)
+    os.replace(tmp, target)
     if verbose:
-        print("built", LIB, file=sys.stderr)
-    return LIB
+        print("built", target, file=sys.stderr)
+    return target
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose=True)
+    # python _build.py [--force] [--lib path.so -DNAME=VAL ...]
+    args = sys.argv[1:]
+    lib = None
+    if "--lib" in args:
+        lib = args[args.index("--lib") + 1]
+    build(force="--force" in args, verbose=True, lib=lib,
+          defines=[a[2:] for a in args if a.startswith("-D")])

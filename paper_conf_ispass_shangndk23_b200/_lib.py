@@ -8,7 +8,8 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libmpspmm.so")
+# MPS_LIB: load another build of the same library (A/B experiments on one GPU box)
+LIB_PATH = os.environ.get("MPS_LIB") or os.path.join(HERE, "libmpspmm.so")
 
 MPS_OK, MPS_ERR_INVALID, MPS_ERR_UNSUPPORTED, MPS_ERR_CUDA, MPS_ERR_WORKSPACE, MPS_ERR_COMM = range(6)
 MPS_FIXUP_AUTO, MPS_FIXUP_ATOMIC, MPS_FIXUP_CARRY = 0, 1, 2

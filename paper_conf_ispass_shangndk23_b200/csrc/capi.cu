@@ -3,6 +3,7 @@
 #include <cstdio>
 #include <cstring>
 #include <cstdarg>
+#include <cstdlib>
 #include <vector>
 
 #include "mps_internal.cuh"
@@ -50,8 +51,8 @@ struct Vec {
     int tile = 0;  // columns per launch (multiple of 32*W)
 };
 
-// Widest lane vector the alignment of B and C allows, preferring widths that fill the
-// 32 lanes of the warp; V = ceil(K_tile / (32 W)) <= 4 slots per lane.
+// Widest lane vector (16 B when possible) that the alignment of B and C allows.  Rows
+// narrower than 32*W columns are gathered NR at a time per warp instruction.
 Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C, int64_t ldc) {
     const int eb = elt_bytes(dt);
     const int cand_f32[3] = {4, 2, 1};
@@ -63,13 +64,31 @@ Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C
         return K % W == 0 && ldb % W == 0 && ((uintptr_t)B % (size_t)(W * eb)) == 0 &&
                ldc % cw == 0 && ((uintptr_t)C % (size_t)(cw * 4)) == 0;
     };
+    // MPS_MAX_W: debug/tuning cap on the lane vector width (elements)
+    static const int max_w = [] {
+        const char *e = getenv("MPS_MAX_W");
+        return e ? atoi(e) : 16;
+    }();
     Vec v;
     for (int i = 0; i < nc && v.tile == 0; ++i)
-        if (ok(cand[i]) && K >= 32 * cand[i]) { v.W = cand[i]; v.tile = 32 * cand[i] * 4; }
-    for (int i = 0; i < nc && v.tile == 0; ++i)
-        if (ok(cand[i])) { v.W = cand[i]; v.tile = 32 * cand[i] * 4; }
+        if (cand[i] <= max_w && ok(cand[i])) { v.W = cand[i]; v.tile = 32 * cand[i] * 4; }
     if (v.tile == 0) { v.W = 1; v.tile = 128; }
     return v;
+}
+
+// Lane geometry of one column tile of kt columns: V slots per lane, NR rows per warp
+// instruction (NR > 1 only when a row needs fewer than 32 lanes).
+void tile_geometry(int32_t kt, int W, int *V, int *NR) {
+    const int lanes = (kt + W - 1) / W;
+    if (lanes >= 32) {
+        *NR = 1;
+        *V = (kt + 32 * W - 1) / (32 * W);
+    } else {
+        int lr = 1;
+        while (lr < lanes) lr <<= 1;
+        *NR = 32 / lr;
+        *V = 1;
+    }
 }
 
 mps_status check_csr(const mps_csr *A, bool device_ptrs_needed = true) {
@@ -131,8 +150,14 @@ mps_status run_segments(mps::SegArgs base, int32_t dt, int32_t K, const Vec &v, 
         a.kpad = (int32_t)carry_kpad(K, v);
         // TMA staging needs col and val equally aligned modulo 16 B
         a.direct = ((((uintptr_t)base.col) ^ ((uintptr_t)base.val)) & 15u) != 0;
-        const int V = (kt + 32 * v.W - 1) / (32 * v.W);
-        MPS_CUDA(mps::launch_segments(a, dt, v.W, V, fix, s), "segment kernel");
+        static const int hints = [] {
+            const char *e = getenv("MPS_L2_HINTS");
+            return e ? atoi(e) : 1;
+        }();
+        a.l2_hints = hints;
+        int V, NR;
+        tile_geometry(kt, v.W, &V, &NR);
+        MPS_CUDA(mps::launch_segments(a, dt, v.W, V, NR, fix, s), "segment kernel");
         if (fix == mps::FIX_CARRY) MPS_CUDA(mps::launch_carry_reduce(a, s), "carry reduce");
     }
     return MPS_OK;

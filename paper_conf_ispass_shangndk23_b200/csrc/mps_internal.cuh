@@ -40,6 +40,7 @@ struct SegArgs {
     int32_t kpad;
     int64_t nnz_end;    // one past the last readable (global) nnz index of col/val
     int32_t direct;     // 1: col/val misaligned relative to each other -> no TMA staging
+    int32_t l2_hints;   // 1: B evict_last / col,val evict_first; 0: evict_normal everywhere
 };
 
 // Host launchers (defined in the .cu files).
@@ -51,7 +52,7 @@ cudaError_t launch_zero_split(const int32_t *rp, int32_t m, const int32_t *cx,
                               const int32_t *cy, int64_t P, float *C, int64_t ldc,
                               int64_t row_base, int32_t K, int32_t tail_row, float *tail,
                               cudaStream_t s);
-cudaError_t launch_segments(const SegArgs &a, int b_dtype, int W, int V, int fix,
+cudaError_t launch_segments(const SegArgs &a, int b_dtype, int W, int V, int NR, int fix,
                             cudaStream_t s);
 cudaError_t launch_carry_reduce(const SegArgs &a, cudaStream_t s);
 cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx, int32_t n,
@@ -82,6 +83,11 @@ __device__ __forceinline__ float ld_stream_f32(const float *p) {
 __device__ __forceinline__ uint64_t policy_evict_last() {
     uint64_t p;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_normal() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
 __device__ __forceinline__ uint64_t policy_evict_first() {

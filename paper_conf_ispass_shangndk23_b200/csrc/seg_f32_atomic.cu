@@ -1,0 +1,8 @@
+// seg_f32_atomic.cu -- instantiations of the segment kernel for B = float, atomic fix-up.
+#include "segment.cuh"
+
+namespace mps {
+cudaError_t launch_segments_f32_atomic(const SegArgs &a, int W, int V, int NR, cudaStream_t s) {
+    return dispatch_w<float, FIX_ATOMIC>(a, W, V, NR, s);
+}
+}  // namespace mps

@@ -1,0 +1,425 @@
+#pragma once
+#include <cstdlib>
+// segment.cuh -- a3 (+ a4 partial rows): the merge-path segment kernel template (Alg. 2,
+// PAPER.md P:100-131, sec. III-B/C P:121-147).  Instantiated per (B dtype, fix-up) in
+// seg_*.cu so the build parallelises.
+//
+// B200 mapping (replaces the paper's thread-to-SIMD-lane mapping of sec. III-C,
+// P:137-147, with the same intent: fill every lane with useful dimensions):
+//  * one merge-path segment per warp (the paper's "thread");
+//  * each lane gathers W consecutive elements of a B row with one vector load
+//    (float4 / bf16x8 = 16 B); LR = 32/NR lanes cover a row of K <= 32*W columns, so one
+//    warp instruction gathers NR different non-zeros of the segment (K=64 fp32: NR=2;
+//    K=16: NR=8; K >= 128: NR=1 and V = K/(32W) slots per lane).  The NR partial sums
+//    of a row are combined with a warp-shuffle butterfly only when the row ends;
+//  * the segment's contiguous col/val range is staged through shared memory by 1-D TMA
+//    bulk copies (cp.async.bulk + mbarrier), double-buffered in chunks of kCH non-zeros
+//    per warp, one chunk ahead across the warp's segments;
+//  * the nnz stream is flat: U independent gathers are issued before any is consumed,
+//    regardless of where rows end; a batch wholly inside the current row takes a
+//    check-free fast path (gathers + packed FFMA2);
+//  * complete rows: one streaming vector store (Alg. 2 line 15); partial rows (lines 5,
+//    9, 13): one vector red.global.add per W floats (atomic mode) or a record in the
+//    workspace (carry mode, settled by carry_reduce_kernel).
+#include "mps_internal.cuh"
+
+namespace mps {
+
+#ifndef MPS_CHUNK
+#define MPS_CHUNK 256
+#endif
+constexpr int kCH = MPS_CHUNK;     // non-zeros per staged chunk (per warp)
+constexpr int kSegMinBlocks = 3;   // 24 resident warps/SM (<= 80 registers)
+
+struct __align__(16) WarpStage {
+    int32_t col[2][kCH];
+    float val[2][kCH];
+};
+
+// element e (runtime, < 4) of a 4-vector, as selects (no local-memory indexing)
+__device__ __forceinline__ int pick4(const int4 &v, int e) {
+    const int lo = (e & 1) ? v.y : v.x, hi = (e & 1) ? v.w : v.z;
+    return (e & 2) ? hi : lo;
+}
+__device__ __forceinline__ float pick4f(const float4 &v, int e) {
+    const float lo = (e & 1) ? v.y : v.x, hi = (e & 1) ? v.w : v.z;
+    return (e & 2) ? hi : lo;
+}
+
+// registers: 80 (3 CTAs/SM) unless a lane holds > 8 words of B per gather (K > 256 fp32)
+template <int W, int V, typename TB>
+constexpr int seg_min_blocks() {
+    return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2 : kSegMinBlocks;
+}
+
+template <int W, int V, int NR, typename TB, int FIX>
+__global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB>()))
+segment_kernel(const SegArgs a) {
+    using BV = BVec<TB, W>;
+    using raw_t = typename BV::raw;
+    static_assert(NR == 1 || V == 1, "several rows per instruction only for one slot");
+    constexpr int LR = 32 / NR;                          // lanes per B row
+    constexpr int kWarps = kBlock / 32;
+    constexpr int kWords = (W * (int)sizeof(TB) + 3) / 4;
+    // per-lane gathers per batch: ~4 KB of B rows in flight per warp
+    constexpr int UL0 = (V * kWords >= 8) ? 4 : ((V * kWords >= 4) ? 8 : 16);
+    constexpr int UL = (UL0 * NR > 32) ? (32 / NR > 0 ? 32 / NR : 1) : UL0;
+    constexpr int U = UL * NR;                           // non-zeros per batch
+    static_assert(kCH % U == 0, "chunk must hold whole batches");
+
+    __shared__ WarpStage stage[kWarps];
+    __shared__ uint64_t bars[kWarps][2];
+
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    const int grp = NR == 1 ? 0 : lane / LR;  // which of the NR non-zeros of an instruction
+    const int lr = lane % LR;      // lane inside the row
+    WarpStage &st = stage[warp];
+    if (lane == 0) {
+        mbar_init(&bars[warp][0], 1);
+        mbar_init(&bars[warp][1], 1);
+    }
+    mbar_fence_init();
+    __syncthreads();
+
+    const uint64_t pol_last = a.l2_hints ? policy_evict_last() : policy_evict_normal();
+    const uint64_t pol_first = a.l2_hints ? policy_evict_first() : policy_evict_normal();
+    const int64_t wid = (int64_t)blockIdx.x * kWarps + warp;
+    const int64_t wstride = (int64_t)gridDim.x * kWarps;
+
+    const int32_t *__restrict__ rp = a.rp;
+    const int32_t *__restrict__ col = a.col;
+    const float *__restrict__ val = a.val;
+    const char *__restrict__ Bc = reinterpret_cast<const char *>(a.B);
+    const uint32_t ldb_bytes = (uint32_t)(a.ldb * (int64_t)sizeof(TB));
+    const int m = a.m;
+    const bool direct = a.direct != 0;
+
+    int cofs[V];
+    bool act[V];
+    const char *bl[V];  // this lane's slot inside B row 0 (column 0 if inactive)
+#pragma unroll
+    for (int s = 0; s < V; ++s) {
+        cofs[s] = (s * LR + lr) * W;
+        act[s] = cofs[s] < a.K;
+        bl[s] = Bc + (act[s] ? cofs[s] * (int)sizeof(TB) : 0);
+    }
+    const bool writer = grp == 0;  // after the butterfly, group 0 writes the row
+
+    // chunk origin of a segment: nnz index whose col address is 16-B aligned (TMA) or
+    // simply ys rounded down to a multiple of 4 (direct mode)
+    auto seg_origin = [&](int ys) -> int {
+        if (direct) return ys & ~3;
+        return ys - (int)(((uintptr_t)(col + ys) & 15u) >> 2);
+    };
+    // TMA may not read past the last 16-B boundary inside [.., nnz_end)
+    const int64_t lim4 = a.nnz_end - (int64_t)(((uintptr_t)(col + a.nnz_end) & 15u) >> 2);
+
+    // ---------------- producer: one chunk ahead, across this warp's segments ----------
+    int64_t pseg = wid;
+    int pys = 0, pye = 0, psb = 0, pk = 0, pnch = 0, pbuf = 0;
+    auto prod_load_seg = [&]() {
+        if (pseg < a.P) {
+            pys = __ldg(a.cy + pseg);
+            pye = __ldg(a.cy + pseg + 1);
+            psb = seg_origin(pys);
+            pnch = pye > pys ? (pye - psb + kCH - 1) / kCH : 0;
+        }
+        pk = 0;
+    };
+    auto produce = [&]() {
+        while (pseg < a.P && pk >= pnch) {
+            pseg += wstride;
+            prod_load_seg();
+        }
+        if (pseg >= a.P) return;
+        const int cb = psb + pk * kCH;
+        const int hi = min(pye, cb + kCH);
+        int32_t *dc = st.col[pbuf];
+        float *dv = st.val[pbuf];
+        if (!direct) {
+            int64_t ce = cb + (((int64_t)hi - cb + 3) & ~3ll);
+            if (ce > lim4) ce = lim4 > cb ? lim4 : cb;
+            const uint32_t bytes = (uint32_t)(ce - cb) * 4u;
+            if (lane == 0) {
+                fence_proxy_async_smem();
+                mbar_arrive_expect_tx(&bars[warp][pbuf], 2u * bytes);
+                if (bytes) {
+                    tma_load_1d(dc, col + cb, bytes, &bars[warp][pbuf], pol_first);
+                    tma_load_1d(dv, val + cb, bytes, &bars[warp][pbuf], pol_first);
+                }
+            }
+            const int rem = hi - (int)ce;   // < 4 entries at the very end of the array
+            if (lane < rem) {
+                dc[ce - cb + lane] = col[ce + lane];
+                dv[ce - cb + lane] = val[ce + lane];
+            }
+        } else {
+            for (int t = lane; cb + t < hi; t += 32) {
+                if (cb + t >= pys) {
+                    dc[t] = __ldg(col + cb + t);
+                    dv[t] = __ldg(val + cb + t);
+                }
+            }
+        }
+        ++pk;
+        pbuf ^= 1;
+    };
+    prod_load_seg();
+    produce();
+
+    uint32_t phase0 = 0, phase1 = 0;
+    int cbuf = 0;
+
+    for (int64_t seg = wid; seg < a.P; seg += wstride) {
+        const int xs = __ldg(a.cx + seg), ys = __ldg(a.cy + seg);
+        const int xe = __ldg(a.cx + seg + 1), ye = __ldg(a.cy + seg + 1);
+        const int sb = seg_origin(ys);
+        const int nch = ye > ys ? (ye - sb + kCH - 1) / kCH : 0;
+
+        // row_ptr window: lane l holds rp[wb + l]
+        int wb = xs;
+        int win = (wb + lane <= m) ? __ldg(rp + wb + lane) : 0x7fffffff;
+        const int rp_xs = __shfl_sync(0xffffffffu, win, 0);
+        int rend = __shfl_sync(0xffffffffu, win, 1);   // rp[r + 1]
+        int rbeg = rp_xs;                               // rp[r]
+        const bool start_in = xs < m && ys > rp_xs;     // Alg. 2 line 2 (start_nz != 0)
+        int r = xs;
+
+        float acc[V][W];
+#pragma unroll
+        for (int s = 0; s < V; ++s)
+#pragma unroll
+            for (int w = 0; w < W; ++w) acc[s][w] = 0.f;
+
+        // sum the NR partial accumulators of the row (warp-shuffle butterfly)
+        auto combine = [&]() {
+            if constexpr (NR > 1) {
+#pragma unroll
+                for (int off = LR; off < 32; off <<= 1)
+#pragma unroll
+                    for (int s = 0; s < V; ++s)
+#pragma unroll
+                        for (int w = 0; w < W; ++w)
+                            acc[s][w] += __shfl_xor_sync(0xffffffffu, acc[s][w], off);
+            }
+        };
+        auto write_row = [&](float *dst, bool atomic) {
+            if (writer) {
+#pragma unroll
+                for (int s = 0; s < V; ++s)
+                    if (act[s]) {
+                        if (atomic) CVec<W>::add(dst + cofs[s], acc[s]);
+                        else CVec<W>::store(dst + cofs[s], acc[s]);
+                    }
+            }
+        };
+
+        // Row r ends inside this segment: settle it and move to row r + 1.
+        auto finish_row = [&]() {
+            combine();
+            if (r == xs && start_in) {
+                // partial start row (Alg. 2 lines 8-9): atomic, or carry record slot 0
+                if (FIX == FIX_ATOMIC) {
+                    if (ys < rend)
+                        write_row((r == a.tail_row) ? a.tail
+                                                    : a.C + ((int64_t)r - a.row_base) * a.ldc,
+                                  true);
+                } else {
+                    write_row(a.rec + (seg * 2) * (int64_t)a.kpad, false);
+                }
+            } else {
+                // complete row (line 15): plain store, no initialisation of C needed
+                write_row(a.C + ((int64_t)r - a.row_base) * a.ldc, false);
+            }
+#pragma unroll
+            for (int s = 0; s < V; ++s)
+#pragma unroll
+                for (int w = 0; w < W; ++w) acc[s][w] = 0.f;
+            ++r;
+            int idx = r + 1 - wb;
+            if (idx >= 32) {
+                wb = r;
+                win = (wb + lane <= m) ? __ldg(rp + wb + lane) : 0x7fffffff;
+                idx = 1;
+            }
+            rbeg = rend;
+            rend = __shfl_sync(0xffffffffu, win, idx);
+        };
+
+        auto fma_row = [&](float v, const raw_t (&b)[V]) {
+#pragma unroll
+            for (int s = 0; s < V; ++s) {
+                float f[W];
+                BV::cvt(b[s], f);
+                if constexpr (W == 1) {
+                    acc[s][0] = fmaf(v, f[0], acc[s][0]);
+                } else {
+#pragma unroll
+                    for (int w = 0; w < W; w += 2) fma2(acc[s][w], acc[s][w + 1], v, f[w], f[w + 1]);
+                }
+            }
+        };
+
+        for (int k = 0; k < nch; ++k) {
+            if (!direct) {
+                mbar_wait(&bars[warp][cbuf], cbuf ? phase1 : phase0);
+                if (cbuf) phase1 ^= 1u; else phase0 ^= 1u;
+            }
+            __syncwarp();
+            produce();                  // next chunk into the other buffer
+            if (direct) __syncwarp();
+            const int cb = sb + k * kCH;
+            const int32_t *sc = st.col[cbuf];
+            const float *sv = st.val[cbuf];
+            int q = ys - cb;
+            q = q > 0 ? (q / U) * U : 0;
+            const int qend = min(kCH, ye - cb);
+            for (; q < qend; q += U) {
+                const int j0 = cb + q;
+                raw_t bv[UL][V];
+                const bool full = j0 >= ys && j0 + U <= ye;
+                // my non-zeros of this batch: u = i*NR + grp (i < UL).  Column indices
+                // and values are read as broadcast 16-B LDS of 4 consecutive entries
+                // (NR <= 4) and each lane selects its own; branch-free: outside the
+                // segment the column index is clamped to 0 (a harmless in-bounds row).
+                uint32_t cid[UL];
+                if constexpr (NR <= 4) {
+#pragma unroll
+                    for (int t = 0; t < U / 4; ++t) {
+                        const int4 c4 = *reinterpret_cast<const int4 *>(sc + q + 4 * t);
+#pragma unroll
+                        for (int k = 0; k < 4 / NR; ++k)
+                            cid[t * (4 / NR) + k] =
+                                (uint32_t)(NR == 1 ? pick4(c4, k) : pick4(c4, k * NR + grp));
+                    }
+                } else {
+#pragma unroll
+                    for (int i = 0; i < UL; ++i) cid[i] = (uint32_t)sc[q + i * NR + grp];
+                }
+                if (!full) {
+#pragma unroll
+                    for (int i = 0; i < UL; ++i) {
+                        const int j = j0 + i * NR + grp;
+                        cid[i] = (j >= ys && j < ye) ? cid[i] : 0u;
+                    }
+                }
+#pragma unroll
+                for (int i = 0; i < UL; ++i)
+#pragma unroll
+                    for (int s = 0; s < V; ++s)
+                        bv[i][s] = BV::load(reinterpret_cast<const TB *>(
+                                                row_addr(bl[s], cid[i], ldb_bytes)), pol_last);
+
+                if (full && j0 + U <= rend) {
+                    // fast path: U non-zeros of the current row, no checks
+                    if constexpr (NR <= 4) {
+#pragma unroll
+                        for (int t = 0; t < U / 4; ++t) {
+                            const float4 v4 = *reinterpret_cast<const float4 *>(sv + q + 4 * t);
+#pragma unroll
+                            for (int k = 0; k < 4 / NR; ++k)
+                                fma_row(NR == 1 ? pick4f(v4, k) : pick4f(v4, k * NR + grp),
+                                        bv[t * (4 / NR) + k]);
+                        }
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < UL; ++i) fma_row(sv[q + i * NR + grp], bv[i]);
+                    }
+                } else {
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        const int j = j0 + u;
+                        if (j >= ys && j < ye) {
+                            while (j >= rend) finish_row();
+                            if (NR == 1 || grp == u % NR) fma_row(sv[q + u], bv[u / NR]);
+                        }
+                    }
+                }
+            }
+            cbuf ^= 1;
+        }
+        // rows whose end item lies in this segment after its last non-zero
+        while (r < xe) finish_row();
+
+        // r == xe: the segment's non-zeros of row xe, if any (lines 3-5 / 11-13)
+        if (xe < m && ye > rbeg) {
+            combine();
+            const bool single = (xs == xe) && start_in;
+            if (FIX == FIX_ATOMIC)
+                write_row((xe == a.tail_row) ? a.tail : a.C + ((int64_t)xe - a.row_base) * a.ldc,
+                          true);
+            else
+                write_row(a.rec + (seg * 2 + (single ? 0 : 1)) * (int64_t)a.kpad, false);
+        }
+    }
+}
+
+template <int W, int V, int NR, typename TB, int FIX>
+static cudaError_t launch_seg(const SegArgs &a, cudaStream_t s) {
+    static int blocks_per_sm = 0;
+    if (blocks_per_sm == 0) {
+        // the staging buffers need the large shared-memory carveout for
+        // seg_min_blocks() CTAs per SM; without the hint the driver may pick a smaller one
+        // MPS_CARVEOUT: shared-memory carveout hint in percent (-1: none)
+        static const int carve = [] {
+            const char *e = getenv("MPS_CARVEOUT");
+            return e ? atoi(e) : -1;
+        }();
+        cudaError_t e = cudaSuccess;
+        if (carve >= 0) {
+            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX>,
+                                     cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+            if (e != cudaSuccess) return e;
+        }
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX>, kBlock, 0);
+        if (e != cudaSuccess) return e;
+        if (blocks_per_sm < 1) blocks_per_sm = 1;
+    }
+    const int64_t warps_per_block = kBlock / 32;
+    int64_t need = (a.P + warps_per_block - 1) / warps_per_block;
+    const int64_t cap = (int64_t)blocks_per_sm * num_sms();
+    const int64_t grid = need < cap ? need : cap;
+    if (grid <= 0) return cudaSuccess;
+    segment_kernel<W, V, NR, TB, FIX><<<(unsigned)grid, kBlock, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+// (W, V, NR) dispatch.  NR > 1 only with V == 1.
+template <typename TB, int FIX, int W>
+static cudaError_t dispatch_v(const SegArgs &a, int V, int NR, cudaStream_t s) {
+    if (V == 1) {
+        switch (NR) {
+        case 1: return launch_seg<W, 1, 1, TB, FIX>(a, s);
+        case 2: return launch_seg<W, 1, 2, TB, FIX>(a, s);
+        case 4: return launch_seg<W, 1, 4, TB, FIX>(a, s);
+        case 8: return launch_seg<W, 1, 8, TB, FIX>(a, s);
+        case 16: return launch_seg<W, 1, 16, TB, FIX>(a, s);
+        case 32: return launch_seg<W, 1, 32, TB, FIX>(a, s);
+        default: return cudaErrorInvalidValue;
+        }
+    }
+    if (NR != 1) return cudaErrorInvalidValue;
+    switch (V) {
+    case 2: return launch_seg<W, 2, 1, TB, FIX>(a, s);
+    case 3: return launch_seg<W, 3, 1, TB, FIX>(a, s);
+    case 4: return launch_seg<W, 4, 1, TB, FIX>(a, s);
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+template <typename TB, int FIX>
+static cudaError_t dispatch_w(const SegArgs &a, int W, int V, int NR, cudaStream_t s) {
+    switch (W) {
+    case 1: return dispatch_v<TB, FIX, 1>(a, V, NR, s);
+    case 2: return dispatch_v<TB, FIX, 2>(a, V, NR, s);
+    case 4: return dispatch_v<TB, FIX, 4>(a, V, NR, s);
+    case 8:
+        if constexpr (sizeof(TB) == 2) return dispatch_v<TB, FIX, 8>(a, V, NR, s);
+        return cudaErrorInvalidValue;
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+}  // namespace mps
