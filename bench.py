@@ -240,14 +240,15 @@ def main():
         L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt_code, P, fix, ctypes.byref(nb))
         ws = torch.empty(max(nb.value, 1), dtype=torch.uint8, device=dev)
         tiles = -(-K // 512) if args.dtype == "f32" else -(-K // 1024)
-        launches_per_step = 1 + (1 if fix != L.MPS_FIXUP_CARRY else 0) + \
-            tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1)
+        launches_per_step = 1 + tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1)
 
         def step(ev=None):
-            L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx), _p(cy),
-                            s_ptr)
-            if fix != L.MPS_FIXUP_CARRY:
-                L.mps_zero_split_rows(ctypes.byref(a), _p(cx), _p(cy), P, _p(C), K, K, s_ptr)
+            if fix != L.MPS_FIXUP_CARRY:   # a2 + zeroing of the cut rows, one launch
+                L.mps_partition_split(_p(A.row_ptr), g.m, g.nnz, P, Lp, _p(cx), _p(cy), _p(C),
+                                      K, K, s_ptr)
+            else:
+                L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx),
+                                _p(cy), s_ptr)
             if ev is not None:
                 ev[0].record(stream)
             L.mps_spmm_segments(ctypes.byref(a), _p(Bd), dt_code, K, K, _p(C), K, _p(cx),

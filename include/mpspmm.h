@@ -73,8 +73,10 @@ const char *mps_last_error(void);
 /* a1 -- schedule sizing (host only, no GPU needed).  Alg. 1 lines 2-3 and
  * sec. III-C: M = m + nnz; P = max(ceil(M / cost), min_parts);
  * L = ceil(M / P) (reading R1).  items_per_part (the paper's merge-path cost,
- * P:137) == 0 selects the library default for (K, b_dtype); min_parts (the paper's
- * thread threshold) == 0 selects the library default.  Outputs P and L.    */
+ * P:137) == 0 selects the library default, tuned on B200 by average row length:
+ * clamp(next_pow2(4 * ceil(nnz/m)), 1024, 2048) items per warp segment; min_parts
+ * (the paper's thread threshold) == 0 selects 1184 (8 per SM of 148).
+ * Outputs P and L.                                                                */
 mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
                     int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out);
 
@@ -86,6 +88,15 @@ mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t 
 mps_status mps_partition(const int32_t *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
                          int64_t diag_end, int64_t num_parts, int64_t items_per_part,
                          int32_t *coord_x, int32_t *coord_y, void *stream);
+
+/* a2 + the atomic fix-up's precondition in ONE launch: mps_partition, and every row cut
+ * by one of the diagonals (x_p < m, y_p > row_ptr[x_p]) gets its K floats of C zeroed
+ * (C row r at C + r*ldc).  Equivalent to mps_partition followed by mps_zero_split_rows
+ * (reading R10).  Asynchronous on stream.                                          */
+mps_status mps_partition_split(const int32_t *row_ptr, int64_t m, int64_t nnz,
+                               int64_t num_parts, int64_t items_per_part, int32_t *coord_x,
+                               int32_t *coord_y, float *C, int64_t ldc, int32_t K,
+                               void *stream);
 
 /* a3+a4 -- offline SpMM with a precomputed schedule (computed once, reused).
  * C = A * B; C is overwritten entirely (it need not be initialised: complete rows

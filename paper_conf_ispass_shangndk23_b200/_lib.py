@@ -39,6 +39,7 @@ _SIGS = {
     "mps_last_error": [],
     "mps_plan": [_i64, _i64, _i32, _i32, _i64, _i64, _p, _p],
     "mps_partition": [_p, _i64, _i64, _i64, _i64, _i64, _i64, _p, _p, _p],
+    "mps_partition_split": [_p, _i64, _i64, _i64, _i64, _p, _p, _p, _i64, _i32, _p],
     "mps_spmm_workspace_bytes": [_p, _i32, _i32, _i64, _i32, _p],
     "mps_spmm": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _p, _sz, _p],
     "mps_zero_split_rows": [_p, _p, _p, _i64, _p, _i64, _i32, _p],

@@ -37,13 +37,18 @@ inline size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
 inline int elt_bytes(int32_t dt) { return dt == MPS_DT_BF16 ? 2 : 4; }
 
-// Default merge-path cost (items per warp segment) by feature width; the paper tunes
-// this per K (Fig. 6); these are B200 values.
-int64_t default_cost(int32_t K, int32_t dt) {
+// Default merge-path cost (items per warp segment).  The paper tunes this per K on an
+// RTX 6000 (Fig. 6: 15-50 items per thread).  On B200 the measured
+// optimum (profiles/r01/cost_sweep.md) follows the average row length rather than K:
+// ~4 rows per segment, clamped to [1024, 2048] items (Reddit avg 492 -> 2048; products
+// avg 50 and R-MAT avg 16 -> 1024).
+int64_t default_cost(int64_t m, int64_t nnz, int32_t K, int32_t dt) {
+    (void)K;
     (void)dt;
-    if (K <= 32) return 256;
-    if (K <= 128) return 512;
-    return 256;
+    const int64_t avg = m > 0 ? (nnz + m - 1) / m : 1;
+    int64_t c = 1;
+    while (c < 4 * avg) c <<= 1;
+    return c < 1024 ? 1024 : (c > 2048 ? 2048 : c);
 }
 
 struct Vec {
@@ -206,7 +211,7 @@ mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t 
     if (b_dtype != MPS_DT_F32 && b_dtype != MPS_DT_BF16)
         return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", b_dtype);
     if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
-    const int64_t cost = items_per_part ? items_per_part : default_cost(K, b_dtype);
+    const int64_t cost = items_per_part ? items_per_part : default_cost(m, nnz, K, b_dtype);
     const int64_t pmin = min_parts ? min_parts : kDefaultMinParts;
     const int64_t M = m + nnz;                      // Alg. 1 line 2
     int64_t P = (M + cost - 1) / cost;              // threads = merge_items / cost
@@ -228,6 +233,22 @@ mps_status mps_partition(const int32_t *row_ptr, int64_t m, int64_t nnz, int64_t
     MPS_CUDA(mps::launch_partition(row_ptr, m, nnz, diag_begin, diag_end - diag_begin, num_parts,
                                    items_per_part, coord_x, coord_y, nullptr, 0, 0, 0, -1,
                                    nullptr, (cudaStream_t)stream),
+             "partition kernel");
+    return MPS_OK;
+}
+
+mps_status mps_partition_split(const int32_t *row_ptr, int64_t m, int64_t nnz,
+                               int64_t num_parts, int64_t items_per_part, int32_t *coord_x,
+                               int32_t *coord_y, float *C, int64_t ldc, int32_t K,
+                               void *stream) {
+    if (m < 0 || nnz < 0 || num_parts < 1 || items_per_part < 0 || K < 0 || (K > 0 && ldc < K))
+        return fail(MPS_ERR_INVALID, "bad partition sizes");
+    if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (!row_ptr || !coord_x || !coord_y || (K > 0 && m > 0 && !C))
+        return fail(MPS_ERR_INVALID, "NULL pointer");
+    MPS_CUDA(mps::launch_partition(row_ptr, m, nnz, 0, m + nnz, num_parts, items_per_part, coord_x,
+                                   coord_y, K > 0 ? C : nullptr, ldc, 0, K, -1, nullptr,
+                                   (cudaStream_t)stream),
              "partition kernel");
     return MPS_OK;
 }
@@ -492,9 +513,10 @@ mps_status mps_shard_bounds(const int32_t *row_ptr_host, int64_t m, int64_t nnz,
     return MPS_OK;
 }
 
-static mps_status shard_plan(const int32_t *X, const int32_t *Y, int32_t rank, int32_t K,
-                             int32_t dt, int64_t ipp, int64_t minp, int64_t *P, int64_t *L,
-                             int64_t *D0, int64_t *span) {
+static mps_status shard_plan(const mps_csr *A, const int32_t *X, const int32_t *Y,
+                             int32_t rank, int32_t K, int32_t dt, int64_t ipp, int64_t minp,
+                             int64_t *P, int64_t *L, int64_t *D0, int64_t *span) {
+    if (ipp == 0) ipp = default_cost(A->m, A->nnz, K, dt);  // the whole graph's row length
     *D0 = (int64_t)X[rank] + Y[rank];
     const int64_t D1 = (int64_t)X[rank + 1] + Y[rank + 1];
     *span = D1 - *D0;
@@ -516,7 +538,8 @@ mps_status mps_spmm_shard_workspace_bytes(const mps_csr *A, int32_t K, int32_t b
     const int64_t M = A->m + A->nnz;
     const int64_t span = (M + world - 1) / world;
     int64_t P, L;
-    if ((st = mps_plan(span, 0, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
+    const int64_t ipp = items_per_part ? items_per_part : default_cost(A->m, A->nnz, K, b_dtype);
+    if ((st = mps_plan(span, 0, K, b_dtype, ipp, min_parts, &P, &L))) return st;
     Vec vmin;
     vmin.W = 1;
     vmin.tile = 128;
@@ -543,7 +566,7 @@ mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int6
     cudaStream_t s = (cudaStream_t)stream;
     MPS_CUDA(cudaMemsetAsync(tail_out, 0, (size_t)K * 4, s), "zero tail");
     int64_t P, L, D0, span;
-    if ((st = shard_plan(X, Y, rank, K, b_dtype, items_per_part, min_parts, &P, &L, &D0, &span)))
+    if ((st = shard_plan(A, X, Y, rank, K, b_dtype, items_per_part, min_parts, &P, &L, &D0, &span)))
         return st;
     if (span == 0) return MPS_OK;
     const int fix = resolve_fix(fixup);

@@ -74,6 +74,28 @@ def test_partition_bit_exact_random_and_subranges():
         assert np.array_equal(cx.cpu().numpy(), ox) and np.array_equal(cy.cpu().numpy(), oy)
 
 
+def test_partition_split_zeroes_exactly_cut_rows():
+    rs = np.random.RandomState(4)
+    for trial in range(20):
+        g = rand_graph(rs, int(rs.randint(1, 300)), 40, 9, seed=trial)
+        A = dev(g)
+        P = int(rs.randint(1, 60))
+        L = -(-(g.m + g.nnz) // P)
+        K = 7
+        C = torch.full((g.m, K + 3), float("nan"), device="cuda")
+        cx = torch.empty(P + 1, dtype=torch.int32, device="cuda")
+        cy = torch.empty_like(cx)
+        M.mps_partition_split(api._p(A.row_ptr), g.m, g.nnz, P, L, api._p(cx), api._p(cy),
+                              api._p(C), K + 3, K, api._stream())
+        ox, oy = O.partition(g.row_ptr, P, L)
+        assert np.array_equal(cx.cpu().numpy(), ox) and np.array_equal(cy.cpu().numpy(), oy)
+        cut = sorted({int(ox[p]) for p in range(P + 1) if ox[p] < g.m and oy[p] > g.row_ptr[ox[p]]})
+        Ch = C.cpu().numpy()
+        zeroed = sorted(np.nonzero(~np.isnan(Ch[:, :K]).any(axis=1))[0].tolist())
+        assert zeroed == cut
+        assert np.all(Ch[cut, :K] == 0) and np.isnan(Ch[:, K:]).all()
+
+
 def test_partition_fig3():
     rp = np.array([0, 8, 12, 13, 14, 15, 15, 16, 16, 16, 16], np.int32)
     g = G.random_csr(10, 10, np.diff(rp).astype(np.int32), 1)
