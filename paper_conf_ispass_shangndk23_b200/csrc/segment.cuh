@@ -47,9 +47,19 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 }
 
 // registers: 80 (3 CTAs/SM) unless a lane holds > 8 words of B per gather (K > 256 fp32)
+#ifndef MPS_MINB_BF16
+#define MPS_MINB_BF16 2   // measured: bf16 variants spill at 80 registers (profiles/r01)
+#endif
+#ifndef MPS_MINB_F32
+#define MPS_MINB_F32 3
+#endif
+#ifndef MPS_UL_DIV
+#define MPS_UL_DIV 1
+#endif
 template <int W, int V, typename TB>
 constexpr int seg_min_blocks() {
-    return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2 : kSegMinBlocks;
+    return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2
+                                                      : (sizeof(TB) == 2 ? MPS_MINB_BF16 : MPS_MINB_F32);
 }
 
 template <int W, int V, int NR, typename TB, int FIX>
@@ -62,7 +72,8 @@ segment_kernel(const SegArgs a) {
     constexpr int kWarps = kBlock / 32;
     constexpr int kWords = (W * (int)sizeof(TB) + 3) / 4;
     // per-lane gathers per batch: ~4 KB of B rows in flight per warp
-    constexpr int UL0 = (V * kWords >= 8) ? 4 : ((V * kWords >= 4) ? 8 : 16);
+    constexpr int UL00 = (V * kWords >= 8) ? 4 : ((V * kWords >= 4) ? 8 : 16);
+    constexpr int UL0 = (sizeof(TB) == 2 && UL00 / MPS_UL_DIV >= 2) ? UL00 / MPS_UL_DIV : UL00;
     constexpr int UL = (UL0 * NR > 32) ? (32 / NR > 0 ? 32 / NR : 1) : UL0;
     constexpr int U = UL * NR;                           // non-zeros per batch
     static_assert(kCH % U == 0, "chunk must hold whole batches");
@@ -327,13 +338,23 @@ segment_kernel(const SegArgs a) {
                         for (int i = 0; i < UL; ++i) fma_row(sv[q + i * NR + grp], bv[i]);
                     }
                 } else {
+                    // slow path: the batch crosses row ends (or the segment's edges).
+                    // One pass per row intersecting the batch: predicated FMAs for the
+                    // non-zeros of the current row, then settle the row.
+                    float vl[UL];
 #pragma unroll
-                    for (int u = 0; u < U; ++u) {
-                        const int j = j0 + u;
-                        if (j >= ys && j < ye) {
-                            while (j >= rend) finish_row();
-                            if (NR == 1 || grp == u % NR) fma_row(sv[q + u], bv[u / NR]);
+                    for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
+                    int jc = j0 > ys ? j0 : ys;                  // next non-zero to consume
+                    const int jend = (j0 + U < ye) ? j0 + U : ye;
+                    while (jc < jend) {
+                        while (jc >= rend) finish_row();          // rows ending before jc
+                        const int lim = rend < jend ? rend : jend;  // row r's part: [jc, lim)
+#pragma unroll
+                        for (int i = 0; i < UL; ++i) {
+                            const int j = j0 + i * NR + grp;
+                            if (j >= jc && j < lim) fma_row(vl[i], bv[i]);
                         }
+                        jc = lim;
                     }
                 }
             }

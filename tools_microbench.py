@@ -9,15 +9,19 @@ from paper_conf_ispass_shangndk23_b200.api import _p, _stream
 
 wl = sys.argv[1] if len(sys.argv) > 1 else "reddit"
 K = int(sys.argv[2]) if len(sys.argv) > 2 else 64
+dt = sys.argv[3] if len(sys.argv) > 3 else "f32"
 g = G.workload(wl); B = torch.from_numpy(G.features(wl, K)).cuda()
+if dt == "bf16":
+    B = B.to(torch.bfloat16)
+DT = 1 if dt == "bf16" else 0
 A = M.CSR.from_numpy(g.row_ptr, g.col_idx, g.val, g.n)
 a = A.struct(); s = _stream()
-P, Lp = M.plan(g.m, g.nnz, K)
+P, Lp = M.plan(g.m, g.nnz, K, DT)
 cx = torch.empty(P + 1, dtype=torch.int32, device="cuda"); cy = torch.empty_like(cx)
 C = torch.empty(g.m, K, device="cuda")
 L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx), _p(cy), s)
 def seg():
-    L.mps_spmm_segments(ctypes.byref(a), _p(B), 0, K, K, _p(C), K, _p(cx), _p(cy), P, 1, None, 0, s)
+    L.mps_spmm_segments(ctypes.byref(a), _p(B), DT, K, K, _p(C), K, _p(cx), _p(cy), P, 1, None, 0, s)
 def zero():
     L.mps_zero_split_rows(ctypes.byref(a), _p(cx), _p(cy), P, _p(C), K, K, s)
 def timeit(fn, pre=None, n=6):
