@@ -49,6 +49,11 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--out", default="")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="N > 1 process-group backend (gloo: CPU-staged tails, for testing "
+                         "several ranks on one GPU)")
+    ap.add_argument("--cuda-graph", action="store_true",
+                    help="capture each step in a CUDA graph and replay it (launch-bound graphs)")
     ap.add_argument("--flush", default="write", choices=["write", "read", "none"],
                     help="L2 flush before each timed step: write (default) or read a 2x-L2 "
                          "buffer, or none")
@@ -193,11 +198,14 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+    ngpu = torch.cuda.device_count()
+    dev = torch.device("cuda", local % ngpu)   # several ranks may share a GPU (gloo tests)
     torch.cuda.set_device(dev)
+    if world > 1:
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
 
     name = args.workload
     K = args.K or G.WORKLOADS[name][3][0]
@@ -271,7 +279,7 @@ def main():
             sh.local(Bd)
             if ev is not None:
                 ev[1].record(stream)
-            tails = M.exchange_tails(sh.tail, world)
+            tails = M.exchange_tails(sh.tail, world)      # the path's one collective
             sh.settle(tails)
         units_nnz = g.nnz
         units_rows = g.m
@@ -286,10 +294,25 @@ def main():
         step()
     torch.cuda.synchronize(dev)
 
+    run_step = step
+    if args.cuda_graph and world == 1:
+        cg = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(cg):
+            step()
+        torch.cuda.synchronize(dev)
+
+        def run_step(ev=None):            # events cannot split a replay: time the graph
+            if ev is not None:
+                ev[0].record(stream)
+            cg.replay()
+            if ev is not None:
+                ev[1].record(stream)
+        stream = torch.cuda.current_stream(dev)
+
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
             torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
            for _ in range(args.steps)]
-    clocks = ClockSampler(local)
+    clocks = ClockSampler(dev.index)
     clocks.start()
     time.sleep(0.3)
     barrier()
@@ -298,7 +321,7 @@ def main():
     for i in range(args.steps):
         do_flush()                        # L2 flush between timed steps (not timed)
         evs[i][0].record(stream)
-        step((evs[i][1], evs[i][2]))
+        run_step((evs[i][1], evs[i][2]))
         evs[i][3].record(stream)
     torch.cuda.synchronize(dev)
     barrier()
@@ -404,6 +427,7 @@ def main():
                        "read": "flushed before every timed step (2x L2 read, untimed)",
                        "none": "not flushed (col/val > L2)"}[args.flush],
                 "parallelism": "merge-path shards x%d" % world, "graph_sha": g.digest(),
+                "cuda_graph": bool(args.cuda_graph and world == 1),
                 "gen_s": round(gen_s, 2),
             },
             "effective_gbs": eff_gbs,

@@ -7,9 +7,9 @@ entry points one to one; ``api`` and ``sharded`` marshal torch tensors to them.
 """
 from . import _lib
 from ._lib import *  # noqa: F401,F403  (mps_* entry points, MpsError, constants)
-from .api import (CSR, Schedule, mps_csr_host, partition, plan, spmm, spmm_host,  # noqa: F401
+from .api import (CSR, CapturedSpMM, Schedule, mps_csr_host, partition, plan, spmm, spmm_host,  # noqa: F401
                   validate_csr, write_stats)
 from .sharded import ShardedSpMM, exchange_tails, shard_bounds  # noqa: F401
 
-__all__ = ["CSR", "Schedule", "plan", "partition", "spmm", "spmm_host", "write_stats",
+__all__ = ["CSR", "CapturedSpMM", "Schedule", "plan", "partition", "spmm", "spmm_host", "write_stats",
            "validate_csr", "ShardedSpMM", "shard_bounds", "exchange_tails"] + list(_lib.EXPORTED)

@@ -143,6 +143,41 @@ def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomi
     return C
 
 
+class CapturedSpMM:
+    """The online path (mps_spmm_online: partition + zeroing + segment kernel) captured
+    once in a CUDA graph for fixed A, B and C buffers, then replayed.  Replay removes
+    the per-call host launch overhead that dominates small graphs (Cora, Pubmed), and
+    keeps the paper's online setting -- the schedule is recomputed on every call
+    (P:151).  Update B / A values in place between replays."""
+
+    def __init__(self, A: CSR, B: torch.Tensor, out: torch.Tensor | None = None,
+                 fixup="atomic", items_per_part=0, min_parts=0):
+        self.A, self.B = A, B
+        self.K = B.shape[1]
+        self.C = torch.empty((A.m, self.K), dtype=torch.float32, device=A.device) \
+            if out is None else out
+        dt = _dtype_code(B)
+        self.a = A.struct()
+        nb = ctypes.c_size_t()
+        L.mps_spmm_online_workspace_bytes(ctypes.byref(self.a), self.K, dt, items_per_part,
+                                          min_parts, _fix(fixup), ctypes.byref(nb))
+        self.ws = _ws(nb.value, A.device)
+        args = (dt, B.stride(0), self.K, _p(self.C), self.C.stride(0), items_per_part,
+                min_parts, _fix(fixup), _p(self.ws), nb.value)
+
+        def launch():
+            L.mps_spmm_online(ctypes.byref(self.a), _p(self.B), *args, _stream())
+        launch()                      # first call outside capture (occupancy queries)
+        torch.cuda.synchronize(A.device)
+        self.graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(self.graph):
+            launch()
+
+    def __call__(self):
+        self.graph.replay()
+        return self.C
+
+
 def spmm_host(row_ptr, col_idx, val, n_cols, B_host, C_host=None, items_per_part=0,
               min_parts=0, fixup="atomic", device="cuda", stream=None, workspace=None):
     """End to end from HOST buffers (mps_spmm_host): H2D of A and B, online SpMM, D2H

@@ -39,6 +39,13 @@ def exchange_tails(tail: torch.Tensor, world: int, group=None) -> torch.Tensor:
     if world == 1:
         out.copy_(tail.reshape(-1))
         return out
+    if tail.is_cuda and dist.get_backend(group) == "gloo":
+        # gloo has no device all-gather: stage through host memory (test/debug runs only;
+        # production multi-GPU runs use NCCL over NVLink)
+        host = torch.empty(world * tail.numel(), dtype=tail.dtype)
+        dist.all_gather_into_tensor(host, tail.reshape(-1).cpu(), group=group)
+        out.copy_(host)
+        return out
     dist.all_gather_into_tensor(out, tail.reshape(-1).contiguous(), group=group)
     return out
 

@@ -128,6 +128,22 @@ def test_spmm_integer_exact_random(fixup, K):
 
 
 @pytest.mark.parametrize("fixup", ["atomic", "carry"])
+@pytest.mark.parametrize("K", [1, 2, 8, 16, 24, 32, 64, 128, 256, 264, 1032])
+def test_spmm_bf16_integer_exact(fixup, K):
+    """B in {-4..4} is exact in bf16, so the bf16-B path (a5) must match O1 bit-exactly."""
+    rs = np.random.RandomState(100 + K)
+    for trial in range(3):
+        g = rand_graph(rs, int(rs.randint(1, 500)), 200, 12, seed=trial, dup=bool(trial % 2))
+        B = G.dense_int(200, K, seed=trial)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        A = dev(g)
+        for cost in (1, 13, 300, 10 ** 6):
+            C = torch.full((g.m, K), float("nan"), device="cuda")
+            M.spmm(A, tB(B, torch.bfloat16), fixup=fixup, out=C, items_per_part=cost, min_parts=1)
+            assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (trial, cost)
+
+
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
 def test_spmm_padded_and_misaligned(fixup):
     rs = np.random.RandomState(3)
     g = rand_graph(rs, 500, 200, 10, seed=3)
@@ -197,6 +213,24 @@ def test_spmm_tolerance_workloads(name, K, fixup):
         M.spmm(A, tB(B), fixup=fixup, out=C, items_per_part=cost)
         r = O.check(C.cpu().numpy(), ref, bnd)
         assert r["ok"], r
+
+
+def test_captured_graph_replay():
+    g = G.workload("cora")
+    B = G.features("cora", 16)
+    ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B)
+    A = dev(g)
+    Bd = tB(B)
+    cap = M.CapturedSpMM(A, Bd)
+    for _ in range(3):
+        cap.C.fill_(float("nan"))
+        C = cap()
+        torch.cuda.synchronize()
+        assert O.check(C.cpu().numpy(), ref, bnd)["ok"]
+    Bd.mul_(2.0)                               # new B values, same buffer
+    C = cap()
+    torch.cuda.synchronize()
+    assert O.check(C.cpu().numpy(), 2 * ref, 2 * bnd)["ok"]
 
 
 def test_carry_is_deterministic():
