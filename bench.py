@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N > 1 process-group backend (gloo: CPU-staged tails, for testing "
                          "several ranks on one GPU)")
+    ap.add_argument("--hot", default="auto", choices=["auto", "off"],
+                    help="degree-aware L2 residency of B rows (auto: when B exceeds L2/2)")
     ap.add_argument("--cuda-graph", action="store_true",
                     help="capture each step in a CUDA graph and replay it (launch-bound graphs)")
     ap.add_argument("--flush", default="write", choices=["write", "read", "none"],
@@ -249,8 +251,21 @@ def main():
         ws = torch.empty(max(nb.value, 1), dtype=torch.uint8, device=dev)
         tiles = -(-K // 512) if args.dtype == "f32" else -(-K // 1024)
         launches_per_step = 1 + tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1)
+        hot_rows = ctypes.c_int64(-1)
+        if args.hot == "auto":
+            L.mps_hot_budget_rows(ctypes.byref(a), K, dt_code, ctypes.byref(hot_rows))
+        hot_rows = hot_rows.value
+        if hot_rows >= 0:
+            nbh = ctypes.c_size_t()
+            L.mps_hot_rows_workspace_bytes(g.n, ctypes.byref(nbh))
+            hot_ws = torch.empty(max(nbh.value, 1), dtype=torch.uint8, device=dev)
+            hot_bm = torch.empty((g.n + 31) // 32, dtype=torch.int32, device=dev)
+            launches_per_step += 4
 
         def step(ev=None):
+            if hot_rows >= 0:              # hub rows of B -> L2 evict_last (recomputed)
+                L.mps_hot_rows(ctypes.byref(a), hot_rows, _p(hot_bm), _p(hot_ws), nbh.value,
+                               s_ptr)
             if fix != L.MPS_FIXUP_CARRY:   # a2 + zeroing of the cut rows, one launch
                 L.mps_partition_split(_p(A.row_ptr), g.m, g.nnz, P, Lp, _p(cx), _p(cy), _p(C),
                                       K, K, s_ptr)
@@ -259,8 +274,9 @@ def main():
                                 _p(cy), s_ptr)
             if ev is not None:
                 ev[0].record(stream)
-            L.mps_spmm_segments(ctypes.byref(a), _p(Bd), dt_code, K, K, _p(C), K, _p(cx),
-                                _p(cy), P, fix, _p(ws), nb.value, s_ptr)
+            L.mps_spmm_segments_hot(ctypes.byref(a), _p(Bd), dt_code, K, K, _p(C), K, _p(cx),
+                                    _p(cy), P, fix, _p(hot_bm) if hot_rows >= 0 else None,
+                                    _p(ws), nb.value, s_ptr)
             if ev is not None:
                 ev[1].record(stream)
         units_nnz = g.nnz
@@ -428,6 +444,7 @@ def main():
                        "none": "not flushed (col/val > L2)"}[args.flush],
                 "parallelism": "merge-path shards x%d" % world, "graph_sha": g.digest(),
                 "cuda_graph": bool(args.cuda_graph and world == 1),
+                "hot_rows": (hot_rows if world == 1 else None),
                 "gen_s": round(gen_s, 2),
             },
             "effective_gbs": eff_gbs,

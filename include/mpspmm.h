@@ -124,6 +124,31 @@ mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, i
                              const int32_t *coord_y, int64_t num_parts, int32_t fixup,
                              void *workspace, size_t workspace_bytes, void *stream);
 
+/* Degree-aware L2 residency (a B200 addition, not in the paper).  When B does not fit
+ * in L2, the B rows gathered most often (hub columns of a power-law A) should stay in
+ * L2 and the long tail should stream.  mps_hot_rows counts the non-zeros of every
+ * column of A and writes hot_bitmap (caller-owned uint32[(n+31)/32], bit c of word
+ * c/32 set) for the columns with the largest counts such that at most budget_rows rows
+ * are hot (power-of-two count threshold; no host synchronisation).  workspace:
+ * mps_hot_rows_workspace_bytes(n) bytes.  mps_spmm_segments_hot is mps_spmm_segments
+ * with that bitmap: hot rows are gathered with L2 evict_last, the others evict_first.
+ * mps_spmm_online / mps_spmm_host do this automatically when MPS_HOT_FRAC (fraction
+ * of the L2 given to hot rows) is set > 0 and the gathered B exceeds half the L2.
+ * Default off: on B200 the static split gained <= 5% over plain evict_last LRU and
+ * its per-call pre-pass costs more than that online (profiles/r01/hot_rows.md).    */
+mps_status mps_hot_rows_workspace_bytes(int64_t n, size_t *bytes);
+/* The library's choice for (A, K, b_dtype) on the current device: *budget_rows_out =
+ * -1 when B fits in half of the L2 (no hot-row split), else the hot-row budget.     */
+mps_status mps_hot_budget_rows(const mps_csr *A, int32_t K, int32_t b_dtype,
+                               int64_t *budget_rows_out);
+mps_status mps_hot_rows(const mps_csr *A, int64_t budget_rows, uint32_t *hot_bitmap,
+                        void *workspace, size_t workspace_bytes, void *stream);
+mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                 int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                                 const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                                 const uint32_t *hot_bitmap, void *workspace,
+                                 size_t workspace_bytes, void *stream);
+
 /* Online convenience: a1 + a2 + a3 + a4 in one call; the partition is
  * written into the workspace.  items_per_part / min_parts as in mps_plan.         */
 mps_status mps_spmm_online_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,

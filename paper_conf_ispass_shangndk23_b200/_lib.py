@@ -44,6 +44,11 @@ _SIGS = {
     "mps_spmm": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _p, _sz, _p],
     "mps_zero_split_rows": [_p, _p, _p, _i64, _p, _i64, _i32, _p],
     "mps_spmm_segments": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _p, _sz, _p],
+    "mps_hot_rows_workspace_bytes": [_i64, _p],
+    "mps_hot_budget_rows": [_p, _i32, _i32, _p],
+    "mps_hot_rows": [_p, _i64, _p, _p, _sz, _p],
+    "mps_spmm_segments_hot": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _p, _p, _sz,
+                              _p],
     "mps_spmm_online_workspace_bytes": [_p, _i32, _i32, _i64, _i64, _i32, _p],
     "mps_spmm_online": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _p, _sz, _p],
     "mps_spmm_host_workspace_bytes": [_p, _i32, _i32, _i64, _i64, _i64, _i64, _i32, _p],

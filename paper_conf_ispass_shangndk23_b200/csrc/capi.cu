@@ -308,6 +308,15 @@ mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, i
                              int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
                              const int32_t *coord_y, int64_t num_parts, int32_t fixup,
                              void *workspace, size_t workspace_bytes, void *stream) {
+    return mps_spmm_segments_hot(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts,
+                                 fixup, nullptr, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                 int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                                 const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                                 const uint32_t *hot_bitmap, void *workspace,
+                                 size_t workspace_bytes, void *stream) {
     mps_status st = check_csr(A);
     if (st) return st;
     if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
@@ -337,12 +346,71 @@ mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, i
     a.tail_row = -1;
     a.tail = nullptr;
     a.nnz_end = A->nnz;
+    a.hot = hot_bitmap;
     return run_segments(a, b_dtype, K, v, fix, workspace, s);
 }
 
-static size_t online_bytes(int64_t P, int32_t K, const Vec &v, int fix) {
+static size_t hot_scratch_bytes(int64_t n) {
+    return align_up((size_t)n * 4, 256) + align_up(34 * 4, 256);
+}
+static size_t hot_bitmap_bytes(int64_t n) { return align_up((size_t)((n + 31) / 32) * 4, 256); }
+
+mps_status mps_hot_rows_workspace_bytes(int64_t n, size_t *bytes) {
+    if (n < 0 || !bytes) return fail(MPS_ERR_INVALID, "bad arguments");
+    *bytes = hot_scratch_bytes(n);
+    return MPS_OK;
+}
+
+mps_status mps_hot_rows(const mps_csr *A, int64_t budget_rows, uint32_t *hot_bitmap,
+                        void *workspace, size_t workspace_bytes, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (budget_rows < 0 || (A->n > 0 && !hot_bitmap)) return fail(MPS_ERR_INVALID, "bad arguments");
+    if (workspace_bytes < hot_scratch_bytes(A->n) || (A->n > 0 && !workspace))
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes,
+                    hot_scratch_bytes(A->n));
+    if (A->n == 0) return MPS_OK;
+    int32_t *counts = (int32_t *)workspace;
+    uint32_t *hist = (uint32_t *)((char *)workspace + align_up((size_t)A->n * 4, 256));
+    MPS_CUDA(mps::launch_hot_columns(A->col_idx, A->nnz, A->n, budget_rows, counts, hist,
+                                     hot_bitmap, (cudaStream_t)stream),
+             "hot rows");
+    return MPS_OK;
+}
+
+// Use degree-aware L2 residency when the gathered B is larger than half the L2.
+static int64_t hot_budget_rows(const mps_csr *A, int32_t K, int32_t dt) {
+    int dev = 0, l2 = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess ||
+        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev) != cudaSuccess || l2 <= 0)
+        l2 = 126 << 20;
+    const double row = (double)K * elt_bytes(dt);
+    if ((double)A->n * row <= 0.5 * (double)l2) return -1;     // B fits: plain evict_last
+    // Off by default: measured on B200 (profiles/r01/hot_rows.md) the static hub policy
+    // gains <= 5% in the segment kernel and its per-call pre-pass costs more online.
+    static const double frac = [] {
+        const char *e = getenv("MPS_HOT_FRAC");
+        return e ? atof(e) : 0.0;
+    }();
+    if (frac <= 0) return -1;
+    return (int64_t)(frac * (double)l2 / row);
+}
+
+mps_status mps_hot_budget_rows(const mps_csr *A, int32_t K, int32_t b_dtype,
+                               int64_t *budget_rows_out) {
+    mps_status st = check_csr(A, false);
+    if (st) return st;
+    if (!budget_rows_out || K < 0) return fail(MPS_ERR_INVALID, "bad arguments");
+    if (b_dtype != MPS_DT_F32 && b_dtype != MPS_DT_BF16)
+        return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", b_dtype);
+    *budget_rows_out = K > 0 ? hot_budget_rows(A, K, b_dtype) : -1;
+    return MPS_OK;
+}
+
+static size_t online_bytes(int64_t P, int32_t K, const Vec &v, int fix, int64_t n = 0) {
     size_t b = align_up((size_t)(P + 1) * 4, 256) * 2;
     if (fix == mps::FIX_CARRY) b += carry_bytes(P, K, v);
+    if (n > 0) b += hot_bitmap_bytes(n) + hot_scratch_bytes(n);
     return b;
 }
 
@@ -359,7 +427,8 @@ mps_status mps_spmm_online_workspace_bytes(const mps_csr *A, int32_t K, int32_t 
     vmin.tile = 128;
     const Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
     const int fix = resolve_fix(fixup);
-    size_t a = online_bytes(P, K, v, fix), b = online_bytes(P, K, vmin, fix);
+    const int64_t nh = hot_budget_rows(A, K, b_dtype) >= 0 ? A->n : 0;
+    size_t a = online_bytes(P, K, v, fix, nh), b = online_bytes(P, K, vmin, fix, nh);
     *bytes = a > b ? a : b;
     return MPS_OK;
 }
@@ -376,13 +445,23 @@ mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int
     if ((st = mps_plan(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
     const int fix = resolve_fix(fixup);
     const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc);
-    const size_t need = online_bytes(P, K, v, fix);
+    const int64_t hot_rows = hot_budget_rows(A, K, b_dtype);
+    const int64_t nh = hot_rows >= 0 ? A->n : 0;
+    const size_t need = online_bytes(P, K, v, fix, nh);
     if (!workspace || workspace_bytes < need)
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
     cudaStream_t s = (cudaStream_t)stream;
     int32_t *cx = (int32_t *)workspace;
     int32_t *cy = (int32_t *)((char *)workspace + align_up((size_t)(P + 1) * 4, 256));
     void *rec = (char *)workspace + align_up((size_t)(P + 1) * 4, 256) * 2;
+    uint32_t *bitmap = nullptr;
+    if (nh > 0) {
+        char *hb = (char *)workspace + online_bytes(P, K, v, fix, 0);
+        bitmap = (uint32_t *)hb;
+        mps_status hs = mps_hot_rows(A, hot_rows, bitmap, hb + hot_bitmap_bytes(A->n),
+                                     hot_scratch_bytes(A->n), stream);
+        if (hs) return hs;
+    }
     MPS_CUDA(mps::launch_partition(A->row_ptr, A->m, A->nnz, 0, A->m + A->nnz, P, L, cx, cy,
                                    fix == mps::FIX_ATOMIC ? C : nullptr, ldc, 0, K, -1, nullptr,
                                    s),
@@ -403,6 +482,7 @@ mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int
     a.tail_row = -1;
     a.tail = nullptr;
     a.nnz_end = A->nnz;
+    a.hot = bitmap;
     return run_segments(a, b_dtype, K, v, fix, rec, s);
 }
 

@@ -41,6 +41,7 @@ struct SegArgs {
     int64_t nnz_end;    // one past the last readable (global) nnz index of col/val
     int32_t direct;     // 1: col/val misaligned relative to each other -> no TMA staging
     int32_t l2_hints;   // 1: B evict_last / col,val evict_first; 0: evict_normal everywhere
+    const uint32_t *hot; // optional bitmap over B rows: 1 = keep in L2 (evict_last), 0 = stream
 };
 
 // Host launchers (defined in the .cu files).
@@ -61,6 +62,10 @@ cudaError_t launch_write_stats(const int32_t *rp, int32_t m, const int32_t *cx,
                                const int32_t *cy, int64_t P, int64_t *counts, cudaStream_t s);
 cudaError_t launch_validate(const int32_t *rp, const int32_t *col, int64_t m, int64_t n,
                             int64_t nnz, unsigned long long *first_bad, cudaStream_t s);
+
+cudaError_t launch_hot_columns(const int32_t *col, int64_t nnz, int64_t n, int64_t budget_rows,
+                               int32_t *counts, uint32_t *hist, uint32_t *bitmap,
+                               cudaStream_t s);
 
 int num_sms();
 
@@ -96,15 +101,26 @@ __device__ __forceinline__ uint64_t policy_evict_first() {
     return p;
 }
 
-// W consecutive elements of B (type TB) as one raw vector gather (read-only path, no L1
-// allocation, L2 evict_last), converted to fp32 at use.
+// W consecutive elements of B (type TB) as one raw vector gather (read-only path, L2
+// evict_last), converted to fp32 at use.  MPS_B_L1 selects the L1 policy:
+// 0 = no_allocate, 1 = normal allocation, 2 = evict_last (keep hub rows resident).
+#ifndef MPS_B_L1
+#define MPS_B_L1 0
+#endif
+#if MPS_B_L1 == 0
+#define MPS_LDB "ld.global.nc.L1::no_allocate.L2::cache_hint"
+#elif MPS_B_L1 == 1
+#define MPS_LDB "ld.global.nc.L2::cache_hint"
+#else
+#define MPS_LDB "ld.global.nc.L1::evict_last.L2::cache_hint"
+#endif
 template <typename TB, int W> struct BVec;
 
 template <> struct BVec<float, 4> {
     using raw = float4;
     static __device__ __forceinline__ raw load(const float *p, uint64_t pol) {
         raw r;
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+        asm volatile(MPS_LDB ".v4.f32 {%0,%1,%2,%3}, [%4], %5;"
                      : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p), "l"(pol));
         return r;
     }
@@ -116,7 +132,7 @@ template <> struct BVec<float, 2> {
     using raw = float2;
     static __device__ __forceinline__ raw load(const float *p, uint64_t pol) {
         raw r;
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.f32 {%0,%1}, [%2], %3;"
+        asm volatile(MPS_LDB ".v2.f32 {%0,%1}, [%2], %3;"
                      : "=f"(r.x), "=f"(r.y) : "l"(p), "l"(pol));
         return r;
     }
@@ -128,7 +144,7 @@ template <> struct BVec<float, 1> {
     using raw = float;
     static __device__ __forceinline__ raw load(const float *p, uint64_t pol) {
         raw r;
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;"
+        asm volatile(MPS_LDB ".f32 %0, [%1], %2;"
                      : "=f"(r) : "l"(p), "l"(pol));
         return r;
     }
@@ -142,7 +158,7 @@ template <> struct BVec<__nv_bfloat16, 8> {
     using raw = uint4;
     static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
         raw r;
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.b32 {%0,%1,%2,%3}, [%4], %5;"
+        asm volatile(MPS_LDB ".v4.b32 {%0,%1,%2,%3}, [%4], %5;"
                      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
         return r;
     }
@@ -155,7 +171,7 @@ template <> struct BVec<__nv_bfloat16, 4> {
     using raw = uint2;
     static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
         raw r;
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.b32 {%0,%1}, [%2], %3;"
+        asm volatile(MPS_LDB ".v2.b32 {%0,%1}, [%2], %3;"
                      : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
         return r;
     }
@@ -167,7 +183,7 @@ template <> struct BVec<__nv_bfloat16, 2> {
     using raw = uint32_t;
     static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
         raw r;
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;"
+        asm volatile(MPS_LDB ".b32 %0, [%1], %2;"
                      : "=r"(r) : "l"(p), "l"(pol));
         return r;
     }
@@ -179,7 +195,7 @@ template <> struct BVec<__nv_bfloat16, 1> {
     using raw = unsigned short;
     static __device__ __forceinline__ raw load(const __nv_bfloat16 *p, uint64_t pol) {
         raw r;
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b16 %0, [%1], %2;"
+        asm volatile(MPS_LDB ".b16 %0, [%1], %2;"
                      : "=h"(r) : "l"(p), "l"(pol));
         return r;
     }

@@ -105,6 +105,7 @@ segment_kernel(const SegArgs a) {
     const uint32_t ldb_bytes = (uint32_t)(a.ldb * (int64_t)sizeof(TB));
     const int m = a.m;
     const bool direct = a.direct != 0;
+    const uint32_t *__restrict__ hot = a.hot;
 
     int cofs[V];
     bool act[V];
@@ -315,12 +316,27 @@ segment_kernel(const SegArgs a) {
                         cid[i] = (j >= ys && j < ye) ? cid[i] : 0u;
                     }
                 }
+                if (hot == nullptr) {
 #pragma unroll
-                for (int i = 0; i < UL; ++i)
+                    for (int i = 0; i < UL; ++i)
 #pragma unroll
-                    for (int s = 0; s < V; ++s)
-                        bv[i][s] = BV::load(reinterpret_cast<const TB *>(
-                                                row_addr(bl[s], cid[i], ldb_bytes)), pol_last);
+                        for (int s = 0; s < V; ++s)
+                            bv[i][s] = BV::load(reinterpret_cast<const TB *>(
+                                                    row_addr(bl[s], cid[i], ldb_bytes)), pol_last);
+                } else {
+                    // degree-aware L2 residency: hub rows evict_last, the tail streams
+                    uint32_t hw[UL];
+#pragma unroll
+                    for (int i = 0; i < UL; ++i) hw[i] = __ldg(hot + (cid[i] >> 5));
+#pragma unroll
+                    for (int i = 0; i < UL; ++i) {
+                        const uint64_t pol = ((hw[i] >> (cid[i] & 31u)) & 1u) ? pol_last : pol_first;
+#pragma unroll
+                        for (int s = 0; s < V; ++s)
+                            bv[i][s] = BV::load(reinterpret_cast<const TB *>(
+                                                    row_addr(bl[s], cid[i], ldb_bytes)), pol);
+                    }
+                }
 
                 if (full && j0 + U <= rend) {
                     // fast path: U non-zeros of the current row, no checks

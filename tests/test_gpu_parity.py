@@ -233,6 +233,91 @@ def test_captured_graph_replay():
     assert O.check(C.cpu().numpy(), 2 * ref, 2 * bnd)["ok"]
 
 
+def _hot_bitmap(A, budget):
+    import ctypes
+    nb = ctypes.c_size_t()
+    M.mps_hot_rows_workspace_bytes(A.n, ctypes.byref(nb))
+    ws = torch.empty(max(nb.value, 1), dtype=torch.uint8, device="cuda")
+    bm = torch.zeros((A.n + 31) // 32, dtype=torch.int32, device="cuda")
+    a = A.struct()
+    M.mps_hot_rows(ctypes.byref(a), budget, api._p(bm), api._p(ws), nb.value, api._stream())
+    return bm
+
+
+def test_hot_rows_bitmap_rule():
+    g = G.workload("pubmed")
+    A = dev(g)
+    counts = np.bincount(g.col_idx, minlength=g.n)
+    for budget in (0, 10, 500, 5000, 10 ** 6):
+        bm = _hot_bitmap(A, budget).cpu().numpy().view(np.uint32)
+        hot = ((bm[np.arange(g.n) >> 5] >> (np.arange(g.n) & 31)) & 1).astype(bool)
+        # reference rule: smallest power of two t with #{count >= t} <= budget
+        thr = None
+        for b in range(32, 0, -1):
+            t = 1 << (b - 1)
+            if np.count_nonzero(counts >= t) > budget:
+                break
+            thr = t
+        ref = counts >= thr if thr is not None else np.zeros(g.n, bool)
+        assert np.array_equal(hot, ref), budget
+        assert hot.sum() <= budget
+
+
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_spmm_segments_hot_exact(fixup):
+    import ctypes
+    rs = np.random.RandomState(21)
+    for K in (8, 64, 128, 200):
+        g = rand_graph(rs, 700, 300, 12, seed=K)
+        B = G.dense_int(300, K, seed=K)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        A = dev(g)
+        sch = M.Schedule.build(A, K, items_per_part=50, min_parts=1)
+        bm = _hot_bitmap(A, 40)
+        C = torch.full((g.m, K), float("nan"), device="cuda")
+        a = A.struct()
+        Bt = tB(B)
+        nb = ctypes.c_size_t()
+        M.mps_spmm_workspace_bytes(ctypes.byref(a), K, 0, sch.num_parts, api._fix(fixup),
+                                   ctypes.byref(nb))
+        ws = torch.empty(max(nb.value, 1), dtype=torch.uint8, device="cuda")
+        if fixup == "atomic":
+            M.mps_zero_split_rows(ctypes.byref(a), api._p(sch.coord_x), api._p(sch.coord_y),
+                                  sch.num_parts, api._p(C), K, K, api._stream())
+        M.mps_spmm_segments_hot(ctypes.byref(a), api._p(Bt), 0, K, K, api._p(C), K,
+                                api._p(sch.coord_x), api._p(sch.coord_y), sch.num_parts,
+                                api._fix(fixup), api._p(bm), api._p(ws), nb.value, api._stream())
+        assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), K
+
+
+def test_online_hot_path_large_B(monkeypatch):
+    """With MPS_HOT_FRAC set, B larger than half the L2 switches the online path to
+    hot-row residency (the env is read once per process: run this in a subprocess)."""
+    import subprocess, sys, os
+    code = "import sys; sys.path.insert(0, %r); import tests.test_gpu_parity as t; t._online_hot_body()" % \
+        os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, MPS_HOT_FRAC="0.6")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True)
+    assert r.returncode == 0, r.stdout + r.stderr
+
+
+def _online_hot_body():
+    import ctypes
+    n, K = 300000, 256                          # 307 MB of fp32 B
+    rl = np.random.RandomState(3).randint(0, 8, size=n).astype(np.int32)
+    g = G.random_csr(n, n, rl, 5)
+    A = dev(g)
+    hot = ctypes.c_int64()
+    a = A.struct()
+    M.mps_hot_budget_rows(ctypes.byref(a), K, 0, ctypes.byref(hot))
+    assert hot.value > 0
+    B = G.dense_int(n, K, seed=2)
+    C = M.spmm(A, tB(B))
+    rows = np.random.RandomState(1).choice(n, 2000, replace=False)
+    ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, rows=rows, want_bound=False)
+    assert np.array_equal(C[torch.from_numpy(rows).cuda()].cpu().numpy().astype(np.float64), ref)
+
+
 def test_carry_is_deterministic():
     g = G.workload("pubmed")
     B = tB(G.features("pubmed", 64))
