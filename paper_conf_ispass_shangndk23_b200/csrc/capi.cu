@@ -56,9 +56,25 @@ struct Vec {
     int tile = 0;  // columns per launch (multiple of 32*W)
 };
 
+static int64_t l2_bytes() {
+    static int64_t cache = 0;
+    if (cache == 0) {
+        int dev = 0, l2 = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess ||
+            cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev) != cudaSuccess || l2 <= 0)
+            l2 = 126 << 20;
+        cache = l2;
+    }
+    return cache;
+}
+
 // Widest lane vector (16 B when possible) that the alignment of B and C allows.  Rows
 // narrower than 32*W columns are gathered NR at a time per warp instruction.
-Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C, int64_t ldc) {
+// Column tiling (B200, measured in profiles/r01/tiling.md): when the gathered B (b_rows
+// rows) exceeds half the L2, each pass covers 256-byte slices of the B rows, so the L2
+// holds a larger share of every pass's working set (Reddit K=256 fp32: 8.1 -> 6.5 ms).
+Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C, int64_t ldc,
+               int64_t b_rows = 0) {
     const int eb = elt_bytes(dt);
     const int cand_f32[3] = {4, 2, 1};
     const int cand_bf[4] = {8, 4, 2, 1};
@@ -74,10 +90,27 @@ Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C
         const char *e = getenv("MPS_MAX_W");
         return e ? atoi(e) : 16;
     }();
+    // MPS_MAX_V: debug/tuning cap on slots per lane, i.e. the column-tile width 32*W*V
+    static const int max_v = [] {
+        const char *e = getenv("MPS_MAX_V");
+        const int v = e ? atoi(e) : 4;
+        return v < 1 ? 1 : (v > 4 ? 4 : v);
+    }();
     Vec v;
     for (int i = 0; i < nc && v.tile == 0; ++i)
-        if (cand[i] <= max_w && ok(cand[i])) { v.W = cand[i]; v.tile = 32 * cand[i] * 4; }
-    if (v.tile == 0) { v.W = 1; v.tile = 128; }
+        if (cand[i] <= max_w && ok(cand[i])) { v.W = cand[i]; v.tile = 32 * cand[i] * max_v; }
+    if (v.tile == 0) { v.W = 1; v.tile = 32 * max_v; }
+    // MPS_TILE: tuning override of the column-tile width (0 = rule below, -1 = no tiling)
+    static const int env_tile = [] {
+        const char *e = getenv("MPS_TILE");
+        return e ? atoi(e) : 0;
+    }();
+    int tile = 0;
+    if (env_tile > 0) tile = env_tile;
+    else if (env_tile == 0 && b_rows > 0 &&
+             (double)b_rows * K * eb > 0.5 * (double)l2_bytes())
+        tile = 256 / eb;
+    if (tile > 0 && tile < v.tile && tile < K) v.tile = (tile / v.W > 0 ? tile / v.W : 1) * v.W;
     return v;
 }
 
@@ -324,7 +357,7 @@ mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtyp
     if (K == 0 || A->m == 0) return MPS_OK;
     if (!coord_x || !coord_y) return fail(MPS_ERR_INVALID, "NULL coordinates");
     const int fix = resolve_fix(fixup);
-    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n);
     if (fix == mps::FIX_CARRY && workspace_bytes < carry_bytes(num_parts, K, v))
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes,
                     carry_bytes(num_parts, K, v));
@@ -444,7 +477,7 @@ mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int
     int64_t P, L;
     if ((st = mps_plan(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
     const int fix = resolve_fix(fixup);
-    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n);
     const int64_t hot_rows = hot_budget_rows(A, K, b_dtype);
     const int64_t nh = hot_rows >= 0 ? A->n : 0;
     const size_t need = online_bytes(P, K, v, fix, nh);
@@ -650,7 +683,7 @@ mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int6
         return st;
     if (span == 0) return MPS_OK;
     const int fix = resolve_fix(fixup);
-    const Vec v = choose_vec(K, b_dtype, B, ldb, C_local ? C_local : tail_out, ldc);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C_local ? C_local : tail_out, ldc, A->n);
     const size_t need = online_bytes(P, K, v, fix);
     if (!workspace || workspace_bytes < need)
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
