@@ -3,7 +3,7 @@
 LIBS=$1; CFGS=$2
 for c in $CFGS; do IFS=: read wl k dt <<< "$c"; dt=${dt:-f32}
   for l in $LIBS; do
-    r=$(env $ENVS MPS_LIB=$PWD/paper_conf_ispass_shangndk23_b200/$l python tools_microbench.py $wl $k $dt 2>&1 | tail -1)
+    r=$(env $ENVS MPS_LIB=$PWD/paper_conf_ispass_shangndk23_b200/$l python tools/microbench.py $wl $k $dt 2>&1 | tail -1)
     echo "$wl:$k:$dt $l $r" | cut -c1-150
   done
 done

@@ -15,6 +15,6 @@ if [ "${NCU:-1}" = "1" ]; then
      --log-file gpurun_out/launches_$TAG.csv python bench.py $BENCH_ARGS --steps 3 --warmup 3 \
      --e2e-steps 0 --no-cpu-baseline > gpurun_out/ncu_launch_$TAG.log 2>&1
   for c in ${PROF_CFGS:-reddit:64 reddit:256 products:128 rmat:64}; do
-    ./prof.sh ${TAG}_${c%%:*}_k${c##*:} ${c%%:*} ${c##*:}
+    tools/prof.sh ${TAG}_${c%%:*}_k${c##*:} ${c%%:*} ${c##*:}
   done
 fi

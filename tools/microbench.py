@@ -1,6 +1,6 @@
 """Segment-kernel microbenchmark: back-to-back launches vs. the bench's step order."""
 import ctypes, sys, os, json
-sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch, numpy as np
 import graphgen as G
 import paper_conf_ispass_shangndk23_b200 as M
