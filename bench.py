@@ -190,6 +190,11 @@ def main():
     if args.impl == "reference":
         run_reference(args)
         return
+    world_env = int(os.environ.get("WORLD_SIZE", "1"))
+    if world_env > 1 and "OMP_NUM_THREADS" not in os.environ:
+        # every rank generates the same graph on the host: share the cores
+        local_world = int(os.environ.get("LOCAL_WORLD_SIZE", world_env))
+        os.environ["OMP_NUM_THREADS"] = str(max(1, (os.cpu_count() or 1) // local_world))
     import torch
     import torch.distributed as dist
     import graphgen as G
