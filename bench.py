@@ -287,6 +287,23 @@ def main():
         units_nnz = g.nnz
         units_rows = g.m
     else:
+        # B replication over NVLink (offline, reported separately, not in the step)
+        per = -(-g.n // world)
+        Bmine = Bd[rank * per: min(g.n, (rank + 1) * per)].contiguous()
+        rep_ms = []
+        for _ in range(3):
+            dist.barrier()
+            r0, r1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            r0.record(stream)
+            Brep = M.replicate_B(Bmine, g.n, world)
+            r1.record(stream)
+            torch.cuda.synchronize(dev)
+            rep_ms.append(r0.elapsed_time(r1))
+        assert torch.equal(Brep, Bd)
+        b_rep = torch.tensor([min(rep_ms)], dtype=torch.float64, device=dev)
+        dist.all_reduce(b_rep, op=dist.ReduceOp.MAX)
+        b_rep_ms = float(b_rep[0])
+        del Brep
         sh = M.ShardedSpMM(g.row_ptr, g.col_idx, g.val, g.n, K, rank, world, dev,
                            b_dtype=tdtype, fixup=args.fixup, items_per_part=args.items_per_part,
                            min_parts=args.min_parts)
@@ -465,6 +482,9 @@ def main():
                          "frac": seg_gbs / hbm_peak, "traffic": traffic,
                          "algorithmic_bytes_per_launch": int(seg_bytes),
                          "peak_source": peak_src},
+            "b_replication": ({"ms": b_rep_ms, "bytes_per_rank_received": int(
+                (world - 1) * (-(-g.n // world)) * K * b_elt), "collective": "all_gather_into_tensor",
+                "in_step": False} if world > 1 else None),
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(launches_per_step * args.steps),

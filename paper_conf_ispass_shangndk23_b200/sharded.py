@@ -50,6 +50,28 @@ def exchange_tails(tail: torch.Tensor, world: int, group=None) -> torch.Tensor:
     return out
 
 
+def replicate_B(B_rows: torch.Tensor, n: int, world: int, group=None) -> torch.Tensor:
+    """Replicate B over the ranks (north-star stage 4: "replicates B over NVLink").
+
+    Rank g holds rows [g*ceil(n/G), (g+1)*ceil(n/G)) of B (the last shard padded); one
+    all_gather_into_tensor (NCCL over NVLink/NVSwitch) assembles the full n x K B on
+    every rank.  It runs once per B (offline setting), outside the SpMM step."""
+    per = -(-n // world)
+    K = B_rows.shape[1]
+    shard = torch.zeros((per, K), dtype=B_rows.dtype, device=B_rows.device)
+    shard[: B_rows.shape[0]] = B_rows
+    full = torch.empty((per * world, K), dtype=B_rows.dtype, device=B_rows.device)
+    if world == 1:
+        full.copy_(shard)
+    elif shard.is_cuda and dist.get_backend(group) == "gloo":   # test runs: host staging
+        host = torch.empty(full.shape, dtype=full.dtype)
+        dist.all_gather_into_tensor(host, shard.cpu(), group=group)
+        full.copy_(host)
+    else:
+        dist.all_gather_into_tensor(full, shard, group=group)
+    return full[:n]
+
+
 class ShardedSpMM:
     """Rank-local state of a merge-path sharded SpMM.
 
