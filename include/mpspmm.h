@@ -57,6 +57,11 @@ enum {
 /* Element type of B.  C is always fp32, accumulation always fp32 (reading R15). */
 enum { MPS_DT_F32 = 0, MPS_DT_BF16 = 1 };
 
+/* Fused epilogue applied to C (the GCN layer's sigma; NEXT-3 in SURVEY.md):
+ * RELU stores max(C, 0).  Complete rows get it in the store; rows cut by a schedule
+ * boundary get it after all their partial sums landed.                            */
+enum { MPS_EPI_NONE = 0, MPS_EPI_RELU = 1 };
+
 /* A: m x n CSR.  row_ptr[m+1] (row_ptr[0] = 0, row_ptr[m] = nnz), col_idx[nnz],
  * val[nnz]; columns need not be sorted, duplicates are summed (CSR).        */
 typedef struct {
@@ -149,6 +154,14 @@ mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtyp
                                  const uint32_t *hot_bitmap, void *workspace,
                                  size_t workspace_bytes, void *stream);
 
+/* mps_spmm with a fused epilogue (MPS_EPI_*) and an optional hot-row bitmap (NULL =
+ * none, see mps_hot_rows).  mps_spmm(...) == mps_spmm_ex(..., MPS_EPI_NONE, NULL, ...). */
+mps_status mps_spmm_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                       float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
+                       int64_t num_parts, int32_t fixup, int32_t epilogue,
+                       const uint32_t *hot_bitmap, void *workspace, size_t workspace_bytes,
+                       void *stream);
+
 /* Online convenience: a1 + a2 + a3 + a4 in one call; the partition is
  * written into the workspace.  items_per_part / min_parts as in mps_plan.         */
 mps_status mps_spmm_online_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
@@ -158,6 +171,10 @@ mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int
                            int32_t K, float *C, int64_t ldc, int64_t items_per_part,
                            int64_t min_parts, int32_t fixup, void *workspace,
                            size_t workspace_bytes, void *stream);
+mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                              int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                              int64_t min_parts, int32_t fixup, int32_t epilogue,
+                              void *workspace, size_t workspace_bytes, void *stream);
 
 /* End-to-end call on HOST buffers: copies A and B host->device, runs the online path
  * and copies C device->host, all enqueued on `stream` (pinned host memory gives

@@ -112,8 +112,12 @@ def _ws(nbytes, device):
     return torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=device)
 
 
+EPILOGUE = {"none": L.MPS_EPI_NONE, "relu": L.MPS_EPI_RELU}
+
+
 def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomic",
-         items_per_part=0, min_parts=0, out: torch.Tensor | None = None, stream=None):
+         items_per_part=0, min_parts=0, out: torch.Tensor | None = None, stream=None,
+         epilogue="none"):
     """C = A * B (row-wise product) by MergePath-SpMM.
 
     With ``schedule`` the offline path (mps_spmm) runs; otherwise the online path
@@ -131,15 +135,16 @@ def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomi
         L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt, schedule.num_parts, _fix(fixup),
                                    ctypes.byref(nb))
         ws = _ws(nb.value, A.device)
-        L.mps_spmm(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
-                   _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts, _fix(fixup),
-                   _p(ws), nb.value, st)
+        L.mps_spmm_ex(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
+                      _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts,
+                      _fix(fixup), EPILOGUE[epilogue], None, _p(ws), nb.value, st)
     else:
         L.mps_spmm_online_workspace_bytes(ctypes.byref(a), K, dt, items_per_part, min_parts,
                                           _fix(fixup), ctypes.byref(nb))
         ws = _ws(nb.value, A.device)
-        L.mps_spmm_online(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
-                          items_per_part, min_parts, _fix(fixup), _p(ws), nb.value, st)
+        L.mps_spmm_online_ex(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
+                             items_per_part, min_parts, _fix(fixup), EPILOGUE[epilogue],
+                             _p(ws), nb.value, st)
     return C
 
 

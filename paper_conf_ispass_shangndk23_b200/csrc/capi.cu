@@ -197,6 +197,7 @@ mps_status run_segments(mps::SegArgs base, int32_t dt, int32_t K, const Vec &v, 
         tile_geometry(kt, v.W, &V, &NR);
         MPS_CUDA(mps::launch_segments(a, dt, v.W, V, NR, fix, s), "segment kernel");
         if (fix == mps::FIX_CARRY) MPS_CUDA(mps::launch_carry_reduce(a, s), "carry reduce");
+        else if (a.relu) MPS_CUDA(mps::launch_relu_split(a, s), "relu on cut rows");
     }
     return MPS_OK;
 }
@@ -345,11 +346,47 @@ mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, i
                                  fixup, nullptr, workspace, workspace_bytes, stream);
 }
 
+static mps_status segments_impl(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                                const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                                const uint32_t *hot_bitmap, int32_t relu, void *workspace,
+                                size_t workspace_bytes, void *stream);
+
 mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
                                  int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
                                  const int32_t *coord_y, int64_t num_parts, int32_t fixup,
                                  const uint32_t *hot_bitmap, void *workspace,
                                  size_t workspace_bytes, void *stream) {
+    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                         hot_bitmap, 0, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                       float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
+                       int64_t num_parts, int32_t fixup, int32_t epilogue,
+                       const uint32_t *hot_bitmap, void *workspace, size_t workspace_bytes,
+                       void *stream) {
+    if (epilogue != MPS_EPI_NONE && epilogue != MPS_EPI_RELU)
+        return fail(MPS_ERR_UNSUPPORTED, "epilogue %d", epilogue);
+    if (resolve_fix(fixup) == mps::FIX_ATOMIC) {
+        mps_status st = check_csr(A);
+        if (st) return st;
+        if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
+        if (num_parts < 1) return fail(MPS_ERR_INVALID, "num_parts < 1");
+        if (K == 0 || A->m == 0) return MPS_OK;
+        if ((st = mps_zero_split_rows(A, coord_x, coord_y, num_parts, C, ldc, K, stream)))
+            return st;
+    }
+    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                         hot_bitmap, epilogue == MPS_EPI_RELU, workspace, workspace_bytes,
+                         stream);
+}
+
+static mps_status segments_impl(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                                const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                                const uint32_t *hot_bitmap, int32_t relu, void *workspace,
+                                size_t workspace_bytes, void *stream) {
     mps_status st = check_csr(A);
     if (st) return st;
     if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
@@ -380,6 +417,7 @@ mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtyp
     a.tail = nullptr;
     a.nnz_end = A->nnz;
     a.hot = hot_bitmap;
+    a.relu = relu;
     return run_segments(a, b_dtype, K, v, fix, workspace, s);
 }
 
@@ -470,6 +508,16 @@ mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int
                            int32_t K, float *C, int64_t ldc, int64_t items_per_part,
                            int64_t min_parts, int32_t fixup, void *workspace,
                            size_t workspace_bytes, void *stream) {
+    return mps_spmm_online_ex(A, B, b_dtype, ldb, K, C, ldc, items_per_part, min_parts, fixup,
+                              MPS_EPI_NONE, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                              int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                              int64_t min_parts, int32_t fixup, int32_t epilogue,
+                              void *workspace, size_t workspace_bytes, void *stream) {
+    if (epilogue != MPS_EPI_NONE && epilogue != MPS_EPI_RELU)
+        return fail(MPS_ERR_UNSUPPORTED, "epilogue %d", epilogue);
     mps_status st = check_csr(A);
     if (st) return st;
     if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
@@ -516,6 +564,7 @@ mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int
     a.tail = nullptr;
     a.nnz_end = A->nnz;
     a.hot = bitmap;
+    a.relu = epilogue == MPS_EPI_RELU;
     return run_segments(a, b_dtype, K, v, fix, rec, s);
 }
 

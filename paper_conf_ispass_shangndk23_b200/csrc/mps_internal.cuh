@@ -42,6 +42,8 @@ struct SegArgs {
     int32_t direct;     // 1: col/val misaligned relative to each other -> no TMA staging
     int32_t l2_hints;   // 1: B evict_last / col,val evict_first; 0: evict_normal everywhere
     const uint32_t *hot; // optional bitmap over B rows: 1 = keep in L2 (evict_last), 0 = stream
+    int32_t relu;        // epilogue: 1 = C = max(C, 0) (complete rows at the store; cut rows
+                         // by launch_relu_split after the atomics, or in the carry reduce)
 };
 
 // Host launchers (defined in the .cu files).
@@ -56,6 +58,7 @@ cudaError_t launch_zero_split(const int32_t *rp, int32_t m, const int32_t *cx,
 cudaError_t launch_segments(const SegArgs &a, int b_dtype, int W, int V, int NR, int fix,
                             cudaStream_t s);
 cudaError_t launch_carry_reduce(const SegArgs &a, cudaStream_t s);
+cudaError_t launch_relu_split(const SegArgs &a, cudaStream_t s);
 cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx, int32_t n,
                                float *row, cudaStream_t s);
 cudaError_t launch_write_stats(const int32_t *rp, int32_t m, const int32_t *cx,

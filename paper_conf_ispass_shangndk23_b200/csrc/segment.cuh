@@ -216,13 +216,21 @@ segment_kernel(const SegArgs a) {
                             acc[s][w] += __shfl_xor_sync(0xffffffffu, acc[s][w], off);
             }
         };
-        auto write_row = [&](float *dst, bool atomic) {
+        auto write_row = [&](float *dst, bool atomic, bool relu = false) {
             if (writer) {
 #pragma unroll
                 for (int s = 0; s < V; ++s)
                     if (act[s]) {
-                        if (atomic) CVec<W>::add(dst + cofs[s], acc[s]);
-                        else CVec<W>::store(dst + cofs[s], acc[s]);
+                        if (atomic) {
+                            CVec<W>::add(dst + cofs[s], acc[s]);
+                        } else if (relu) {   // fused epilogue of a complete row
+                            float t[W];
+#pragma unroll
+                            for (int w = 0; w < W; ++w) t[w] = fmaxf(acc[s][w], 0.f);
+                            CVec<W>::store(dst + cofs[s], t);
+                        } else {
+                            CVec<W>::store(dst + cofs[s], acc[s]);
+                        }
                     }
             }
         };
@@ -242,7 +250,7 @@ segment_kernel(const SegArgs a) {
                 }
             } else {
                 // complete row (line 15): plain store, no initialisation of C needed
-                write_row(a.C + ((int64_t)r - a.row_base) * a.ldc, false);
+                write_row(a.C + ((int64_t)r - a.row_base) * a.ldc, false, a.relu != 0);
             }
 #pragma unroll
             for (int s = 0; s < V; ++s)

@@ -65,6 +65,10 @@ carry_reduce_kernel(const SegArgs a) {
             const float4 v = *reinterpret_cast<const float4 *>(a.rec + (s * 2) * (int64_t)a.kpad + c);
             acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
         }
+        if (a.relu) {
+            acc.x = fmaxf(acc.x, 0.f); acc.y = fmaxf(acc.y, 0.f);
+            acc.z = fmaxf(acc.z, 0.f); acc.w = fmaxf(acc.w, 0.f);
+        }
         if (vec) {
             dst[c] = acc.x; dst[c + 1] = acc.y; dst[c + 2] = acc.z; dst[c + 3] = acc.w;
         } else {
@@ -78,6 +82,30 @@ cudaError_t launch_carry_reduce(const SegArgs &a, cudaStream_t s) {
     const int64_t threads = (a.P + 1) * 32;
     const int64_t blocks = (threads + kBlock - 1) / kBlock;
     carry_reduce_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+// Epilogue for the rows cut by a schedule boundary in atomic mode: they are final only
+// after every partial sum has landed, so the ReLU runs here, once per cut row (one warp
+// per first boundary inside the row).
+__global__ void __launch_bounds__(kBlock)
+relu_split_kernel(const SegArgs a) {
+    const int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (p > a.P) return;
+    const int32_t r = a.cx[p];
+    if (r >= a.m || r == a.tail_row) return;
+    const int32_t rs = __ldg(a.rp + r);
+    if (a.cy[p] <= rs) return;
+    if (p > 0 && a.cx[p - 1] == r && a.cy[p - 1] > rs) return;
+    float *dst = a.C + ((int64_t)r - a.row_base) * a.ldc;
+    for (int c = lane; c < a.K; c += 32) dst[c] = fmaxf(dst[c], 0.f);
+}
+
+cudaError_t launch_relu_split(const SegArgs &a, cudaStream_t s) {
+    const int64_t threads = (a.P + 1) * 32;
+    const int64_t blocks = (threads + kBlock - 1) / kBlock;
+    relu_split_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(a);
     return cudaGetLastError();
 }
 

@@ -1,0 +1,47 @@
+"""NEXT-2: two-layer GCN inference on MergePath-SpMM.
+
+    out = A · ( relu( A · (X · W1) ) · W2 )           (A·(X·W) order P:282)
+
+The combination X·W is a plain dense GEMM (cuBLAS through torch.matmul -- a library GEMM,
+not on the SpMM hot path).  The aggregation A·B is MergePath-SpMM (libmpspmm), with the
+layer-1 ReLU fused into it (MPS_EPI_RELU: complete rows at the store, cut rows after
+their partial sums).  ``online=True`` recomputes the merge-path
+schedule on every inference (the paper's online setting) -- one partition per
+inference serves both layers; ``online=False`` computes it once and reuses it for every
+call (the offline default).
+"""
+from __future__ import annotations
+
+import torch
+
+from .api import CSR, Schedule, spmm
+
+
+class GCN2:
+    def __init__(self, A: CSR, W1: torch.Tensor, W2: torch.Tensor, online: bool = False,
+                 b_dtype=torch.float32, fixup: str = "atomic", items_per_part: int = 0,
+                 min_parts: int = 0):
+        self.A, self.W1, self.W2 = A, W1, W2
+        self.online, self.b_dtype, self.fixup = online, b_dtype, fixup
+        self.ipp, self.minp = items_per_part, min_parts
+        self.H = torch.empty((A.m, W1.shape[1]), dtype=torch.float32, device=A.device)
+        self.out = torch.empty((A.m, W2.shape[1]), dtype=torch.float32, device=A.device)
+        # the default plan depends on the graph only, so one schedule serves both layers
+        self.schedule = None if online else Schedule.build(A, W1.shape[1], b_dtype,
+                                                           items_per_part, min_parts)
+
+    def _aggregate(self, B, out, epilogue):
+        return spmm(self.A, B.to(self.b_dtype), schedule=self.schedule, fixup=self.fixup,
+                    items_per_part=self.ipp, min_parts=self.minp, out=out, epilogue=epilogue)
+
+    def layer1(self, X: torch.Tensor) -> torch.Tensor:
+        return self._aggregate(X @ self.W1, self.H, "relu")
+
+    def __call__(self, X: torch.Tensor) -> torch.Tensor:
+        if self.online:
+            # online setting: the schedule is recomputed for every inference --
+            # once, since the default plan depends on the graph only, for both layers
+            self.schedule = Schedule.build(self.A, self.W1.shape[1], self.b_dtype, self.ipp,
+                                           self.minp)
+        H = self.layer1(X)
+        return self._aggregate(H @ self.W2, self.out, "none")

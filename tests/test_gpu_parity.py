@@ -318,6 +318,50 @@ def _online_hot_body():
     assert np.array_equal(C[torch.from_numpy(rows).cuda()].cpu().numpy().astype(np.float64), ref)
 
 
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_relu_epilogue_exact(fixup):
+    """MPS_EPI_RELU == max(A*B, 0) bit-exactly on integer inputs, for complete and cut rows,
+    offline and online, fp32 and bf16 B."""
+    rs = np.random.RandomState(31)
+    for K in (8, 64, 96, 256):
+        g = rand_graph(rs, 600, 200, 14, seed=K)
+        B = G.dense_int(200, K, seed=K)
+        ref = np.maximum(O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False), 0)
+        A = dev(g)
+        for dt in (torch.float32, torch.bfloat16):
+            for cost in (5, 60):
+                sch = M.Schedule.build(A, K, dt, items_per_part=cost, min_parts=1)
+                C = torch.full((g.m, K), float("nan"), device="cuda")
+                M.spmm(A, tB(B, dt), schedule=sch, fixup=fixup, out=C, epilogue="relu")
+                assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (K, dt, cost)
+                C2 = M.spmm(A, tB(B, dt), fixup=fixup, items_per_part=cost, min_parts=1,
+                            epilogue="relu")
+                assert np.array_equal(C2.cpu().numpy().astype(np.float64), ref), (K, dt, cost)
+
+
+@pytest.mark.parametrize("online", [False, True])
+def test_gcn2_layers_against_oracle(online):
+    """2-layer GCN (NEXT-2): each aggregation checked against O1 on the GPU-computed X*W."""
+    g = G.workload("pubmed")
+    A = dev(g)
+    gen = torch.Generator(device="cpu").manual_seed(0)
+    X = torch.randn(g.n, 128, generator=gen).cuda()
+    W1 = (torch.randn(128, 64, generator=gen) / 11).cuda()
+    W2 = (torch.randn(64, 16, generator=gen) / 8).cuda()
+    net = M.GCN2(A, W1, W2, online=online)
+    out = net(X)
+    torch.cuda.synchronize()
+    B1 = (X @ W1).cpu().numpy()
+    ref1, bnd1 = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B1)
+    H = net.H.cpu().numpy()
+    r = O.check(H, np.maximum(ref1, 0), bnd1)
+    assert r["ok"], r
+    B2 = (net.H @ W2).cpu().numpy()
+    ref2, bnd2 = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B2)
+    r = O.check(out.cpu().numpy(), ref2, bnd2)
+    assert r["ok"], r
+
+
 def test_carry_is_deterministic():
     g = G.workload("pubmed")
     B = tB(G.features("pubmed", 64))
