@@ -45,6 +45,8 @@ def _L():
         lib.gen_chung_lu.restype = _p
         lib.gen_rmat.argtypes = [_i32, _i64, _f64, _f64, _f64, _i32, _i64, _u64]
         lib.gen_rmat.restype = _p
+        lib.gen_block_diag.argtypes = [_i64, _i64, _i64, _u64]
+        lib.gen_block_diag.restype = _p
         lib.gen_random_csr.argtypes = [_i64, _i64, _p, _i32, _u64]
         lib.gen_random_csr.restype = _p
         for f in ("gen_rows", "gen_cols", "gen_nnz"):
@@ -97,6 +99,10 @@ def _take(h):
 
 def chung_lu(n, E, alpha, dmax, seed) -> tuple:
     return _take(_L().gen_chung_lu(n, E, alpha, dmax, seed))
+
+
+def block_diag(n, E, block, seed) -> tuple:
+    return _take(_L().gen_block_diag(n, E, block, seed))
 
 
 def rmat(scale, edge_factor, a, b, c, n_evil, evil_len, seed) -> tuple:
@@ -158,9 +164,36 @@ WORKLOADS = {
 }
 
 
+# Table II of the paper: the 22 graphs, shapes only (n, nnz, max degree).
+# Type I (power-law): Chung-Lu with E = nnz//2 undirected edges and the printed max
+# degree as the expected max.  Type II (structured): block-diagonal batches of small
+# graphs (blocks of 32 nodes), locality preserved.  Seeds 1000 + index.
+TABLE2 = [
+    # (name, type, n, nnz, max_degree)
+    ("Cora", 1, 2708, 10556, 168), ("Citeseer", 1, 3327, 9228, 99),
+    ("Pubmed", 1, 19717, 99203, 171), ("Oregon-1", 1, 11492, 46818, 2389),
+    ("As-caida", 1, 31379, 106762, 2628), ("Wiki-Vote", 1, 8297, 103689, 893),
+    ("email-Enron", 1, 36692, 367662, 1383), ("email-Euall", 1, 265214, 420045, 930),
+    ("Nell", 1, 65755, 251550, 4549), ("PPI", 1, 56944, 818716, 429),
+    ("soc-SlashDot811", 1, 77357, 905468, 2508), ("artist", 1, 50515, 1638396, 1469),
+    ("com-Amazon", 1, 334863, 1851744, 549), ("coAuthorsDBLP", 1, 299067, 1955352, 336),
+    ("soc-BlogCatalog", 1, 88784, 2093195, 2538), ("amazon0601", 1, 410236, 4878874, 2760),
+    ("amazon0505", 1, 403394, 5478357, 2760),
+    ("PROTEINS_full", 2, 43466, 162088, 25), ("Twitter-partial", 2, 580768, 1435116, 12),
+    ("DD", 2, 334925, 1686092, 19), ("Yeast", 2, 1710902, 3636546, 6),
+    ("OVCAR-8H", 2, 1889542, 3946402, 5), ("SW-620H", 2, 1888584, 3944206, 5),
+]
+for _i, (_nm, _ty, _n, _nnz, _dmax) in enumerate(TABLE2):
+    WORKLOADS["t2-" + _nm] = ("chung_lu" if _ty == 1 else "block_diag",
+                              dict(n=_n, E=_nnz // 2, dmax=float(_dmax), block=32),
+                              1000 + _i, (16,))
+
+
 def workload(name: str, values: str = "gcn") -> Graph:
     kind, prm, seed, _ = WORKLOADS[name]
-    if kind == "chung_lu":
+    if kind == "block_diag":
+        m, n, rp, ci = block_diag(prm["n"], prm["E"], prm["block"], seed)
+    elif kind == "chung_lu":
         m, n, rp, ci = chung_lu(prm["n"], prm["E"], ALPHA, prm["dmax"], seed)
     else:
         m, n, rp, ci = rmat(prm["scale"], prm["edge_factor"], prm["a"], prm["b"], prm["c"],

@@ -182,6 +182,55 @@ Graph chung_lu(int64_t n, int64_t E, double alpha, double dmax, uint64_t seed) {
     return Graph();
 }
 
+// "Structured" graph (Table II type II: batches of small molecule/protein graphs):
+// block-diagonal, blocks of `block` consecutive nodes, E distinct undirected edges drawn
+// uniformly inside the blocks (first E distinct samples), symmetrised, no self loops.
+// Node ids are NOT permuted: these datasets keep each small graph contiguous.
+Graph block_diag(int64_t n, int64_t E, int64_t block, uint64_t seed) {
+    const int64_t nblk = (n + block - 1) / block;
+    double over = 1.10;
+    for (int attempt = 0; attempt < 8; ++attempt, over *= 1.35) {
+        int64_t Es = (int64_t)((double)E * over) + 64;
+        std::vector<int32_t> u(Es), v(Es);
+#pragma omp parallel for schedule(static)
+        for (int64_t s = 0; s < Es; ++s) {
+            const int64_t b = (int64_t)(rng(seed, S_EDGE, 3 * s) % (uint64_t)nblk);
+            const int64_t lo = b * block, sz = std::min(block, n - lo);
+            u[s] = (int32_t)(lo + (int64_t)(rng(seed, S_EDGE, 3 * s + 1) % (uint64_t)sz));
+            v[s] = (int32_t)(lo + (int64_t)(rng(seed, S_EDGE, 3 * s + 2) % (uint64_t)sz));
+        }
+        // canonical (min, max) keys with the first sample id, sorted and de-duplicated
+        std::vector<std::pair<uint64_t, uint32_t>> key;
+        key.reserve(Es);
+        for (int64_t s = 0; s < Es; ++s)
+            if (u[s] != v[s]) {
+                const uint32_t a = (uint32_t)std::min(u[s], v[s]), b = (uint32_t)std::max(u[s], v[s]);
+                key.push_back({((uint64_t)a << 32) | b, (uint32_t)s});
+            }
+        std::sort(key.begin(), key.end());
+        std::vector<std::pair<uint32_t, uint64_t>> first;   // (sample, edge)
+        for (size_t i = 0; i < key.size(); ++i)
+            if (i == 0 || key[i].first != key[i - 1].first) first.push_back({key[i].second, key[i].first});
+        if ((int64_t)first.size() < E && attempt < 7) continue;
+        if ((int64_t)first.size() > E) {
+            std::nth_element(first.begin(), first.begin() + E, first.end());
+            first.resize(E);
+        }
+        std::vector<int32_t> rows, cols;
+        rows.reserve(2 * first.size());
+        cols.reserve(2 * first.size());
+        for (auto &f : first) {
+            const int32_t a = (int32_t)(f.second >> 32), b = (int32_t)(f.second & 0xffffffffu);
+            rows.push_back(a); cols.push_back(b);
+            rows.push_back(b); cols.push_back(a);
+        }
+        Graph g;
+        build_csr(g, n, n, rows, cols, std::vector<int32_t>(), true);
+        return g;
+    }
+    return Graph();
+}
+
 // R-MAT (Chakrabarti et al.) directed graph, de-duplicated, no self loops, ids
 // permuted; then `n_evil` rows (row 0, row n-1 and seeded-random rows) replaced by
 // `evil_len` distinct columns each ("evil rows").
@@ -264,6 +313,10 @@ void *gen_chung_lu(int64_t n, int64_t E, double alpha, double dmax, uint64_t see
 void *gen_rmat(int32_t scale, int64_t edge_factor, double a, double b, double c, int32_t n_evil,
                int64_t evil_len, uint64_t seed) {
     return new Graph(rmat(scale, edge_factor, a, b, c, n_evil, evil_len, seed));
+}
+
+void *gen_block_diag(int64_t n, int64_t E, int64_t block, uint64_t seed) {
+    return new Graph(block_diag(n, E, block, seed));
 }
 
 // Arbitrary CSR from explicit per-row lengths with uniformly random columns in

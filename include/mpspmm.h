@@ -78,10 +78,11 @@ const char *mps_last_error(void);
 /* a1 -- schedule sizing (host only, no GPU needed).  Alg. 1 lines 2-3 and
  * sec. III-C: M = m + nnz; P = max(ceil(M / cost), min_parts);
  * L = ceil(M / P) (reading R1).  items_per_part (the paper's merge-path cost,
- * P:137) == 0 selects the library default, tuned on B200 by average row length:
- * clamp(next_pow2(4 * ceil(nnz/m)), 1024, 2048) items per warp segment; min_parts
- * (the paper's thread threshold) == 0 selects 1184 (8 per SM of 148).
- * Outputs P and L.                                                                */
+ * P:137) == 0 selects the library default, tuned on B200 (NEXT-1 sweep):
+ * max(64, min(clamp(next_pow2(4*ceil(nnz/m)), 512, 2048),
+ *             pow2_floor(M / (1.5 * resident warps of the current device))))
+ * items per warp segment; min_parts (the paper's thread threshold) == 0
+ * selects 1184 (8 per SM of 148).  Outputs P and L.                               */
 mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
                     int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out);
 

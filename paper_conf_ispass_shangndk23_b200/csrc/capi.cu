@@ -8,6 +8,8 @@
 
 #include "mps_internal.cuh"
 
+namespace mps { int num_sms(); }
+
 namespace {
 
 thread_local char g_err[512] = "";
@@ -38,17 +40,26 @@ inline size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 inline int elt_bytes(int32_t dt) { return dt == MPS_DT_BF16 ? 2 : 4; }
 
 // Default merge-path cost (items per warp segment).  The paper tunes this per K on an
-// RTX 6000 (Fig. 6: 15-50 items per thread).  On B200 the measured
-// optimum (profiles/r01/cost_sweep.md) follows the average row length rather than K:
-// ~4 rows per segment, clamped to [1024, 2048] items (Reddit avg 492 -> 2048; products
-// avg 50 and R-MAT avg 16 -> 1024).
+// RTX 6000 (Fig. 6: 15-50 items per thread).  On B200 the NEXT-1 sweep over
+// the 22 Table-II-shaped graphs and the BASELINE graphs (profiles/r01/sensitivity.md)
+// finds the optimum set by two things rather than K: long rows want long segments
+// (fewer cut rows: ~4 rows per segment, 512..2048 items), and the schedule must keep
+// >= 1.5 waves of resident warps busy, which caps the cost on mid-size graphs:
+//   cost = max(64, min(clamp(next_pow2(4*ceil(nnz/m)), 512, 2048),
+//                      pow2_floor(M / (1.5 * resident_warps))))
+// (geomean 0.974 of the per-graph best on Table II, 0.998 on Reddit/products/R-MAT).
 int64_t default_cost(int64_t m, int64_t nnz, int32_t K, int32_t dt) {
     (void)K;
-    (void)dt;
     const int64_t avg = m > 0 ? (nnz + m - 1) / m : 1;
-    int64_t c = 1;
-    while (c < 4 * avg) c <<= 1;
-    return c < 1024 ? 1024 : (c > 2048 ? 2048 : c);
+    int64_t deg = 1;
+    while (deg < 4 * avg) deg <<= 1;
+    deg = deg < 512 ? 512 : (deg > 2048 ? 2048 : deg);
+    const int64_t resident = (int64_t)mps::num_sms() * (dt == MPS_DT_BF16 ? 16 : 24);
+    const double target = (double)(m + nnz) / (1.5 * (double)resident);
+    int64_t cap = 1;
+    while ((double)(cap * 2) <= target) cap <<= 1;
+    int64_t c = deg < cap ? deg : cap;
+    return c < 64 ? 64 : c;
 }
 
 struct Vec {
