@@ -190,6 +190,15 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
                          int64_t items_per_part, int64_t min_parts, int32_t fixup,
                          void *device_workspace, size_t workspace_bytes, void *stream);
 
+/* NEXT-3: the GCN combination B = X * W (A*(X*W) order) on the sm_100
+ * tensor cores (tcgen05.mma kind::f16, fp32 accumulation in TMEM, TMA-fed), writing B in
+ * bf16 into the row-major layout the SpMM gathers (MPS_DT_BF16, ldb).
+ * X: bf16 [n][ldx] (first F columns used); Wt: bf16 [N][ldw] = W transposed (first F
+ * columns used); B: bf16 [n][ldb].  Requires 16 <= N <= 256, N % 16 == 0, ldx, ldw,
+ * ldb multiples of 8 and 16-B aligned pointers, else MPS_ERR_UNSUPPORTED.           */
+mps_status mps_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
+                       int32_t N, int64_t ldw, void *B, int64_t ldb, void *stream);
+
 /* Fig. 5 statistic: with the Alg. 2 write rules (lines 5, 9, 13 atomic,
  * line 15 regular) for the given schedule, counts_out[0] = #atomic row updates,
  * counts_out[1] = #regular row stores.  counts_out: device int64[2], overwritten. */

@@ -183,6 +183,21 @@ class CapturedSpMM:
         return self.C
 
 
+def xw_bf16(X: torch.Tensor, Wt: torch.Tensor, out: torch.Tensor | None = None, stream=None):
+    """NEXT-3 combination B = X @ W on tcgen05 tensor cores (mps_xw_bf16).
+
+    X: (n, F) bf16 with row stride % 8 == 0; Wt: (N, F) bf16 = W transposed; returns
+    B (n, N) bf16, the row-major layout the SpMM gathers."""
+    assert X.dtype == torch.bfloat16 and Wt.dtype == torch.bfloat16
+    assert X.stride(1) == 1 and Wt.stride(1) == 1 and X.shape[1] == Wt.shape[1]
+    n, F = X.shape
+    N = Wt.shape[0]
+    B = torch.empty((n, N), dtype=torch.bfloat16, device=X.device) if out is None else out
+    L.mps_xw_bf16(_p(X), n, F, X.stride(0), _p(Wt), N, Wt.stride(0), _p(B), B.stride(0),
+                  _stream(stream))
+    return B
+
+
 def spmm_host(row_ptr, col_idx, val, n_cols, B_host, C_host=None, items_per_part=0,
               min_parts=0, fixup="atomic", device="cuda", stream=None, workspace=None):
     """End to end from HOST buffers (mps_spmm_host): H2D of A and B, online SpMM, D2H

@@ -650,6 +650,20 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
     return MPS_OK;
 }
 
+mps_status mps_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
+                       int32_t N, int64_t ldw, void *B, int64_t ldb, void *stream) {
+    if (n < 0 || F < 0 || N < 0 || ldx < F || ldw < F || ldb < N)
+        return fail(MPS_ERR_INVALID, "bad xw sizes");
+    if (n == 0 || N == 0) return MPS_OK;
+    if (!X || !Wt || !B) return fail(MPS_ERR_INVALID, "NULL pointer");
+    const cudaError_t e = mps::launch_xw_bf16(X, n, F, ldx, Wt, N, ldw, B, ldb, (cudaStream_t)stream);
+    if (e == cudaErrorNotSupported)
+        return fail(MPS_ERR_UNSUPPORTED, "xw: need 16 <= N <= 256, N %% 16 == 0, ld %% 8 == 0, "
+                    "16-B aligned pointers");
+    MPS_CUDA(e, "xw gemm");
+    return MPS_OK;
+}
+
 mps_status mps_write_stats(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
                            int64_t num_parts, int64_t *counts_out, void *stream) {
     mps_status st = check_csr(A);

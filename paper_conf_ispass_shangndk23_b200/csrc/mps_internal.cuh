@@ -70,6 +70,9 @@ cudaError_t launch_hot_columns(const int32_t *col, int64_t nnz, int64_t n, int64
                                int32_t *counts, uint32_t *hist, uint32_t *bitmap,
                                cudaStream_t s);
 
+cudaError_t launch_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
+                           int32_t N, int64_t ldw, void *Bout, int64_t ldb, cudaStream_t s);
+
 int num_sms();
 
 // ---------------------------------------------------------------------------------

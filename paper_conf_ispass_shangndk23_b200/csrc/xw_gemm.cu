@@ -1,0 +1,257 @@
+// xw_gemm.cu -- NEXT-3: the GCN combination B = X * W (computed before
+// the aggregation, A*(X*W)) on the 5th-generation tensor cores, writing B in bf16
+// straight into the row-major layout the segment kernel gathers from.
+//
+// One CTA per 128-row tile of X, the whole output width N (<= 256) in TMEM:
+//   warp 0 (one lane): TMA producer -- 2-D tensor loads of X[128 x 64] and Wt[N x 64]
+//                      (bf16, 128-B swizzle) into a 2-4 stage smem ring (mbarrier full/empty),
+//                      sized so that >= 2 CTAs share an SM;
+//   warp 1 (one lane): MMA issuer -- tcgen05.mma.cta_group::1.kind::f16, M=128, N, K=16,
+//                      fp32 accumulator in TMEM; tcgen05.commit frees each stage;
+//   warps 0-3:         epilogue -- tcgen05.ld 32x32b (each thread one row), bf16 convert,
+//                      16-B stores of the B row.
+// The shape is tall and thin (n x F times F x N), so the kernel is HBM-bound on reading X;
+// the tensor cores are far from busy, which is the point: the combination costs one read of
+// X and one write of B.
+#include <cuda.h>
+#include <cuda_bf16.h>
+
+#include "mps_internal.cuh"
+
+namespace mps {
+
+namespace {
+
+constexpr int kXwBM = 128;       // rows of X per CTA (UMMA M)
+constexpr int kXwBK = 64;        // reduction chunk: 64 bf16 = 128 B = one swizzle row
+constexpr int kXwMaxStages = 4;
+constexpr int kXwThreads = 128;
+
+__device__ __forceinline__ uint64_t smem_desc_sw128(uint32_t saddr) {
+    // UMMA shared-memory descriptor, K-major, SWIZZLE_128B (cute::UMMA::SmemDescriptor):
+    // start address >> 4 [0,14); LBO >> 4 [16,30) (unused for swizzled K-major, 1);
+    // SBO >> 4 [32,46) = 1024 B between 8-row core-matrix groups; version 1 [46,48);
+    // base offset 0 (1024-B aligned tiles); layout type 2 = SWIZZLE_128B [61,64).
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+    d |= (uint64_t)1u << 16;
+    d |= (uint64_t)(1024u >> 4) << 32;
+    d |= (uint64_t)1u << 46;
+    d |= (uint64_t)2u << 61;
+    return d;
+}
+
+__device__ __forceinline__ uint32_t instr_desc_bf16(int N) {
+    // kind::f16 instruction descriptor: D fp32 (c_format 1, bits [4,6)), A and B bf16
+    // (a_format 1 bits [7,10), b_format 1 bits [10,13)), both K-major, N >> 3 at [17,23),
+    // M >> 4 at [24,29) with M = 128.
+    return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(kXwBM >> 4) << 24);
+}
+
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map, int c0, int c1,
+                                            uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%2, %3}], [%4];"
+        :: "r"(dst), "l"(map), "r"(c0), "r"(c1), "r"(bar) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait_u32(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred P;\n\t"
+        "XW_WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+        "@!P bra XW_WAIT_%=;\n\t}"
+        :: "r"(bar), "r"(parity) : "memory");
+}
+
+__global__ void __launch_bounds__(kXwThreads)
+xw_gemm_kernel(const __grid_constant__ CUtensorMap map_x, const __grid_constant__ CUtensorMap map_w,
+               int64_t n, int F, int N, int kXwStages, __nv_bfloat16 *__restrict__ Bout,
+               int64_t ldb) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    // 1024-B aligned carve-up: A stages, B stages, then barriers and the TMEM address
+    uint8_t *base = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const uint32_t a_bytes = kXwBM * kXwBK * 2;                       // 16 KB
+    const uint32_t b_bytes = (uint32_t)N * kXwBK * 2;                 // <= 32 KB
+    uint8_t *sA = base;
+    uint8_t *sB = base + kXwStages * a_bytes;
+    uint64_t *full = (uint64_t *)(sB + kXwStages * b_bytes);
+    uint64_t *empty = full + kXwMaxStages;
+    uint64_t *done = empty + kXwMaxStages;
+    uint32_t *tmem_slot = (uint32_t *)(done + 1);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t m0 = (int64_t)blockIdx.x * kXwBM;
+    const int nk = (F + kXwBK - 1) / kXwBK;
+    const uint32_t ncols = N <= 32 ? 32 : (N <= 64 ? 64 : (N <= 128 ? 128 : 256));
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kXwMaxStages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        mbar_init(done, 1);
+        asm volatile("prefetch.tensormap [%0];" :: "l"(&map_x) : "memory");
+        asm volatile("prefetch.tensormap [%0];" :: "l"(&map_w) : "memory");
+    }
+    mbar_fence_init();
+    if (warp == 2) {   // TMEM allocation: one warp, power-of-two columns >= 32
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(smem_u32(tmem_slot)), "r"(ncols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0 && lane == 0) {
+        // ---- TMA producer ----
+        for (int kb = 0; kb < nk; ++kb) {
+            const int s = kb % kXwStages;
+            if (kb >= kXwStages) mbar_wait_u32(smem_u32(&empty[s]), ((kb / kXwStages) - 1) & 1);
+            mbar_arrive_expect_tx(&full[s], a_bytes + b_bytes);
+            tma_load_2d(smem_u32(sA + s * a_bytes), &map_x, kb * kXwBK, (int)m0, smem_u32(&full[s]));
+            tma_load_2d(smem_u32(sB + s * b_bytes), &map_w, kb * kXwBK, 0, smem_u32(&full[s]));
+        }
+    } else if (warp == 1 && lane == 0) {
+        // ---- MMA issuer (single thread) ----
+        const uint32_t idesc = instr_desc_bf16(N);
+        for (int kb = 0; kb < nk; ++kb) {
+            const int s = kb % kXwStages;
+            mbar_wait_u32(smem_u32(&full[s]), (kb / kXwStages) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            const uint64_t da = smem_desc_sw128(smem_u32(sA + s * a_bytes));
+            const uint64_t db = smem_desc_sw128(smem_u32(sB + s * b_bytes));
+#pragma unroll
+            for (int k = 0; k < kXwBK / 16; ++k) {
+                // advance 16 bf16 = 32 B inside the 128-B swizzle row (start address >> 4)
+                const uint64_t a = da + (uint64_t)(k * 2);
+                const uint64_t b = db + (uint64_t)(k * 2);
+                const uint32_t acc = (kb > 0 || k > 0) ? 1u : 0u;
+                asm volatile(
+                    "{\n\t.reg .pred p;\n\t"
+                    "setp.ne.b32 p, %4, 0;\n\t"
+                    "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+                    :: "r"(tmem), "l"(a), "l"(b), "r"(idesc), "r"(acc) : "memory");
+            }
+            // frees the stage once these MMAs have read it
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                         :: "r"(smem_u32(&empty[s])) : "memory");
+        }
+        asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                     :: "r"(smem_u32(done)) : "memory");
+    }
+    __syncwarp();
+
+    // ---- epilogue: TMEM -> registers -> bf16 -> global ----
+    mbar_wait_u32(smem_u32(done), 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const int64_t row = m0 + warp * 32 + lane;
+    for (int c0 = 0; c0 < N; c0 += 32) {
+        uint32_t v[32];
+        const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0;
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+            "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+            "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+            : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
+              "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]),
+              "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]),
+              "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+              "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]),
+              "=r"(v[30]), "=r"(v[31])
+            : "r"(taddr));
+        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+        if (row < n) {
+            const int cols = (N - c0) < 32 ? (N - c0) : 32;   // N % 16 == 0: 16 or 32
+            uint32_t pk[16];
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+                __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * i]),
+                                                         __uint_as_float(v[2 * i + 1]));
+                pk[i] = *reinterpret_cast<uint32_t *>(&h);
+            }
+            uint4 *dst = reinterpret_cast<uint4 *>(Bout + row * ldb + c0);
+            dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+            dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+            if (cols == 32) {
+                dst[2] = make_uint4(pk[8], pk[9], pk[10], pk[11]);
+                dst[3] = make_uint4(pk[12], pk[13], pk[14], pk[15]);
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 2)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;"
+                     :: "r"(tmem), "r"(ncols) : "memory");
+}
+
+using EncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                              const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                              const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                              CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeFn encode_fn() {
+    static EncodeFn fn = nullptr;
+    if (!fn) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) ==
+                cudaSuccess && q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeFn>(p);
+    }
+    return fn;
+}
+
+bool make_map(CUtensorMap *map, const void *ptr, int64_t rows, int64_t cols, int64_t ld_elems,
+              int box_rows) {
+    EncodeFn fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+    const cuuint64_t strides[1] = {(cuuint64_t)ld_elems * 2};
+    const cuuint32_t box[2] = {(cuuint32_t)kXwBK, (cuuint32_t)box_rows};
+    const cuuint32_t estr[2] = {1, 1};
+    return fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(ptr), dims, strides,
+              box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+}  // namespace
+
+// X: bf16 [n][ldx] (F used columns), Wt: bf16 [N][ldw] (= W transposed, F used columns),
+// Bout: bf16 [n][ldb].  Returns cudaErrorNotSupported for shapes the kernel does not cover.
+cudaError_t launch_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
+                           int32_t N, int64_t ldw, void *Bout, int64_t ldb, cudaStream_t s) {
+    if (N < 16 || N > 256 || N % 16 || F < 1 || ldx % 8 || ldw % 8 || ldb % 8 ||
+        ((uintptr_t)X & 15) || ((uintptr_t)Wt & 15) || ((uintptr_t)Bout & 15))
+        return cudaErrorNotSupported;
+    if (n == 0) return cudaSuccess;
+    CUtensorMap mx, mw;
+    if (!make_map(&mx, X, n, F, ldx, kXwBM) || !make_map(&mw, Wt, N, F, ldw, N))
+        return cudaErrorNotSupported;
+    // stages: enough to cover the reduction, but small enough that >= 2 CTAs share an SM
+    // (one CTA's epilogue overlaps another's TMA loads); TMEM: <= 2 x 256 columns per SM.
+    const size_t stage_bytes = (size_t)kXwBM * kXwBK * 2 + (size_t)N * kXwBK * 2;
+    const int nk = (int)((F + kXwBK - 1) / kXwBK);
+    int stages = (int)((100u << 10) / stage_bytes);
+    stages = stages < 2 ? 2 : (stages > kXwMaxStages ? kXwMaxStages : stages);
+    if (stages > nk) stages = nk < 2 ? 2 : nk;
+    const size_t smem = 1024 + (size_t)stages * stage_bytes + 256;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(
+            xw_gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            (int)(1024 + kXwMaxStages * (kXwBM * kXwBK * 2 + 256 * kXwBK * 2) + 256));
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    const unsigned grid = (unsigned)((n + kXwBM - 1) / kXwBM);
+    xw_gemm_kernel<<<grid, kXwThreads, smem, s>>>(mx, mw, n, (int)F, N, stages,
+                                                  reinterpret_cast<__nv_bfloat16 *>(Bout), ldb);
+    return cudaGetLastError();
+}
+
+}  // namespace mps

@@ -14,15 +14,22 @@ from __future__ import annotations
 
 import torch
 
-from .api import CSR, Schedule, spmm
+from .api import CSR, Schedule, spmm, xw_bf16
 
 
 class GCN2:
     def __init__(self, A: CSR, W1: torch.Tensor, W2: torch.Tensor, online: bool = False,
                  b_dtype=torch.float32, fixup: str = "atomic", items_per_part: int = 0,
-                 min_parts: int = 0):
+                 min_parts: int = 0, combination: str = "cublas"):
         self.A, self.W1, self.W2 = A, W1, W2
         self.online, self.b_dtype, self.fixup = online, b_dtype, fixup
+        # "tcgen05": X*W by the library's tensor-core kernel (mps_xw_bf16), B in bf16
+        # straight into the gather layout (NEXT-3); "cublas": torch.matmul
+        self.combination = combination
+        if combination == "tcgen05":
+            self.b_dtype = torch.bfloat16
+            self.W1t = W1.t().contiguous().to(torch.bfloat16)
+            self.W2t = W2.t().contiguous().to(torch.bfloat16)
         self.ipp, self.minp = items_per_part, min_parts
         self.H = torch.empty((A.m, W1.shape[1]), dtype=torch.float32, device=A.device)
         self.out = torch.empty((A.m, W2.shape[1]), dtype=torch.float32, device=A.device)
@@ -34,8 +41,14 @@ class GCN2:
         return spmm(self.A, B.to(self.b_dtype), schedule=self.schedule, fixup=self.fixup,
                     items_per_part=self.ipp, min_parts=self.minp, out=out, epilogue=epilogue)
 
+    def _combine(self, X, W, Wt):
+        if self.combination == "tcgen05":
+            return xw_bf16(X.to(torch.bfloat16), Wt)
+        return X @ W
+
     def layer1(self, X: torch.Tensor) -> torch.Tensor:
-        return self._aggregate(X @ self.W1, self.H, "relu")
+        return self._aggregate(self._combine(X, self.W1, getattr(self, "W1t", None)), self.H,
+                               "relu")
 
     def __call__(self, X: torch.Tensor) -> torch.Tensor:
         if self.online:
@@ -44,4 +57,5 @@ class GCN2:
             self.schedule = Schedule.build(self.A, self.W1.shape[1], self.b_dtype, self.ipp,
                                            self.minp)
         H = self.layer1(X)
-        return self._aggregate(H @ self.W2, self.out, "none")
+        return self._aggregate(self._combine(H, self.W2, getattr(self, "W2t", None)), self.out,
+                               "none")

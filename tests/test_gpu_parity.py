@@ -362,6 +362,32 @@ def test_gcn2_layers_against_oracle(online):
     assert r["ok"], r
 
 
+def test_gcn2_tcgen05_combination():
+    """NEXT-3: X*W on tcgen05 (bf16 B) feeding the SpMM; each stage checked."""
+    g = G.workload("pubmed")
+    A = dev(g)
+    gen = torch.Generator(device="cpu").manual_seed(1)
+    X = torch.randn(g.n, 128, generator=gen).cuda()
+    W1 = (torch.randn(128, 64, generator=gen) / 11).cuda()
+    W2 = (torch.randn(64, 16, generator=gen) / 8).cuda()
+    net = M.GCN2(A, W1, W2, combination="tcgen05")
+    out = net(X)
+    torch.cuda.synchronize()
+    # layer 1: B1 = bf16(X) * bf16(W1) in fp32, rounded to bf16, checked vs fp64
+    Xb, W1b = X.to(torch.bfloat16).double().cpu(), W1.to(torch.bfloat16).double().cpu()
+    B1 = M.xw_bf16(X.to(torch.bfloat16), net.W1t)
+    ref = Xb @ W1b
+    assert torch.all((B1.double().cpu() - ref).abs() <= 2 ** -8 * ref.abs() + 1e-5 * (Xb.abs() @ W1b.abs()))
+    # aggregation on exactly that bf16 B1, with the fused ReLU
+    ref1, bnd1 = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B1.float().cpu().numpy())
+    r = O.check(net.H.cpu().numpy(), np.maximum(ref1, 0), bnd1)
+    assert r["ok"], r
+    B2 = M.xw_bf16(net.H.to(torch.bfloat16), net.W2t)
+    ref2, bnd2 = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B2.float().cpu().numpy())
+    r = O.check(out.cpu().numpy(), ref2, bnd2)
+    assert r["ok"], r
+
+
 def test_carry_is_deterministic():
     g = G.workload("pubmed")
     B = tB(G.features("pubmed", 64))

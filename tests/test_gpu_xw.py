@@ -1,0 +1,52 @@
+"""NEXT-3: the tcgen05 combination kernel B = X*W (mps_xw_bf16) against fp64."""
+import numpy as np
+import pytest
+import torch
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_ispass_shangndk23_b200 as M
+
+
+def _pad(a, ld):
+    out = torch.zeros((a.shape[0], ld), dtype=a.dtype, device=a.device)
+    out[:, : a.shape[1]] = a
+    return out[:, : a.shape[1]]
+
+
+@pytest.mark.parametrize("N", [16, 32, 48, 64, 128, 256])
+@pytest.mark.parametrize("F", [16, 64, 72, 128])
+def test_xw_exact_small_integers(N, F):
+    # |sum| <= F <= 128 < 256: exact in fp32 accumulation AND in the bf16 output
+    g = torch.Generator(device="cpu").manual_seed(N * 1000 + F)
+    n = 1000 + 77                                   # ragged last tile
+    X = torch.randint(-1, 2, (n, F), generator=g).to(torch.bfloat16).cuda()
+    W = torch.randint(-1, 2, (F, N), generator=g).to(torch.bfloat16).cuda()
+    B = M.xw_bf16(X, W.t().contiguous())
+    ref = X.double().cpu() @ W.double().cpu()
+    assert torch.equal(B.double().cpu(), ref)
+
+
+@pytest.mark.parametrize("n,F,N", [(5000, 602, 64), (2000, 100, 256), (129, 1433, 16), (40000, 128, 128)])
+def test_xw_random_within_bf16_rounding(n, F, N):
+    g = torch.Generator(device="cpu").manual_seed(n + F + N)
+    ldx = (F + 7) // 8 * 8                          # TMA needs 16-B row strides
+    X = _pad(torch.randn(n, F, generator=g).to(torch.bfloat16).cuda(), ldx)
+    W = (torch.randn(F, N, generator=g) / F ** 0.5).to(torch.bfloat16)
+    Wt = _pad(W.t().contiguous().cuda(), ldx)
+    B = M.xw_bf16(X, Wt)
+    Xd, Wd = X.double().cpu(), W.double()
+    ref = Xd @ Wd
+    bound = Xd.abs() @ Wd.abs()
+    err = (B.double().cpu() - ref).abs()
+    # bf16 output rounding (unit roundoff 2^-8) + fp32 accumulation of F products
+    assert torch.all(err <= 2.0 ** -8 * ref.abs() + 1e-5 * bound + 1e-30)
+
+
+def test_xw_unsupported_shapes_report_errors():
+    X = torch.zeros((10, 64), dtype=torch.bfloat16, device="cuda")
+    with pytest.raises(M.MpsError):
+        M.xw_bf16(X, torch.zeros((20, 64), dtype=torch.bfloat16, device="cuda"))   # N % 16
+    with pytest.raises(M.MpsError):
+        M.xw_bf16(X, torch.zeros((272, 64), dtype=torch.bfloat16, device="cuda"))  # N > 256

@@ -34,8 +34,9 @@ def main():
         W1 = (torch.randn(F, H, generator=gen) / F ** 0.5).cuda()
         W2 = (torch.randn(H, C, generator=gen) / H ** 0.5).cuda()
         row = {"workload": wl, "n": g.m, "nnz": g.nnz, "F": F, "H": H, "C": C}
-        for mode in ("offline", "online"):
-            net = M.GCN2(A, W1, W2, online=(mode == "online"))
+        for mode in ("offline", "online", "offline_tcgen05"):
+            net = M.GCN2(A, W1, W2, online=(mode == "online"),
+                         combination="tcgen05" if "tcgen05" in mode else "cublas")
             row[mode + "_ms"] = time_it(lambda: net(X))
             g_ = torch.cuda.CUDAGraph()
             net(X); torch.cuda.synchronize()
