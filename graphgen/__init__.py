@@ -213,3 +213,79 @@ def features(name_or_rows, K, seed=None, kind="uniform") -> np.ndarray:
         rows = int(name_or_rows)
         seed = 7 if seed is None else seed
     return dense_uniform(rows, K, seed) if kind == "uniform" else dense_int(rows, K, seed)
+
+
+# --------------------------------------------------------------------------------
+# NEXT-4 "wide" graphs: nnz > 2^31 (int64 row_ptr).  Too large to build on the host and
+# copy per test, so the column and value arrays are a counter-based hash of the global
+# non-zero index j, evaluated either on the device (torch, in chunks) or, for any
+# sampled rows, on the host (numpy) -- the same bytes either way, so the oracle's inputs
+# never come from the device.  splitmix64 finaliser (Steele et al.), logical shifts
+# emulated on torch's signed int64.
+# --------------------------------------------------------------------------------
+_SM_C = (0x9E3779B97F4A7C15, 0xBF58476D1CE4E5B9, 0x94D049BB133111EB)
+
+
+def _s64(c):
+    return c - (1 << 64) if c >= (1 << 63) else c
+
+
+def _mix_np(x):
+    x = np.asarray(x, np.uint64)
+    with np.errstate(over="ignore"):
+        z = x + np.uint64(_SM_C[0])
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(_SM_C[1])
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(_SM_C[2])
+        return z ^ (z >> np.uint64(31))
+
+
+def _mix_torch(x):
+    import torch
+    def srl(v, k):
+        return (v >> k) & ((1 << (64 - k)) - 1)
+    z = x + _s64(_SM_C[0])
+    z = (z ^ srl(z, 30)) * _s64(_SM_C[1])
+    z = (z ^ srl(z, 27)) * _s64(_SM_C[2])
+    return z ^ srl(z, 31)
+
+
+def _h31_np(seed, j):
+    return (_mix_np(_mix_np(np.asarray(j, np.uint64)) ^ np.uint64(seed)) >> np.uint64(33)).astype(np.int64)
+
+
+def _h31_torch(seed, j):
+    z = _mix_torch(_mix_torch(j) ^ int(seed))
+    return (z >> 33) & 0x7FFFFFFF
+
+
+def wide_row_ptr(m, max_len, seed, evil=()) -> np.ndarray:
+    """int64 row_ptr[m+1]: row r has h(seed, r) % (max_len+1) non-zeros, except the
+    (row, length) pairs in ``evil``."""
+    rl = _h31_np(seed, np.arange(m, dtype=np.uint64)) % (max_len + 1)
+    for r, ln in evil:
+        rl[r] = ln
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(rl, out=rp[1:])
+    return rp
+
+
+def wide_cols_vals_host(j, n, seed):
+    """Columns (int32, uniform in [0, n)) and integer values {1,2,3} (fp32) of the
+    global non-zeros j (numpy int64 array)."""
+    j = np.asarray(j, np.int64)
+    col = (_h31_np(seed + 1, j.astype(np.uint64)) % n).astype(np.int32)
+    val = (1 + _h31_np(seed + 2, j.astype(np.uint64)) % 3).astype(np.float32)
+    return col, val
+
+
+def wide_cols_vals_device(nnz, n, seed, device="cuda", chunk=1 << 27):
+    """The same arrays as wide_cols_vals_host over j = 0..nnz-1, built on the device."""
+    import torch
+    col = torch.empty(nnz, dtype=torch.int32, device=device)
+    val = torch.empty(nnz, dtype=torch.float32, device=device)
+    for j0 in range(0, nnz, chunk):
+        j = torch.arange(j0, min(nnz, j0 + chunk), dtype=torch.int64, device=device)
+        col[j0:j0 + j.numel()] = (_h31_torch(seed + 1, j) % n).to(torch.int32)
+        val[j0:j0 + j.numel()] = (1 + _h31_torch(seed + 2, j) % 3).to(torch.float32)
+        del j
+    return col, val

@@ -238,6 +238,48 @@ mps_status mps_apply_tails(const float *tails, const int32_t *X, const int32_t *
                            int32_t world, int32_t rank, int32_t K, float *C_local,
                            int64_t ldc, void *stream);
 
+/* NEXT-4 -- 64-bit non-zero indices, for graphs with
+ * M = m + nnz >= 2^31 (the paper motivates billion-edge graphs).  Rows and
+ * columns stay below 2^31, so coord_x and col_idx stay int32; row_ptr and the nnz
+ * coordinate y are int64.  The method is unchanged: the same a1-a4 steps run with
+ * 64-bit y (x = max{x : x + row_ptr[x] <= d} on int64 diagonals d).
+ * A: row_ptr int64[m+1], col_idx int32[nnz], val fp32[nnz]; m, n < 2^31,
+ * nnz < 2^62, else MPS_ERR_UNSUPPORTED.  Every other convention (ownership, streams,
+ * errors, overwrite of C, fix-up modes, epilogues) is that of the int32 calls above:
+ *   mps_plan64           = mps_plan without the 2^31 limit on M;
+ *   mps_partition64      = mps_partition, coord_y int64[num_parts+1];
+ *   mps_spmm64           = mps_spmm_ex (no hot-row bitmap), coord_y int64;
+ *   mps_spmm64_online    = mps_spmm_online_ex;
+ *   mps_write_stats64, mps_validate_csr64 = mps_write_stats, mps_validate_csr.      */
+typedef struct {
+    int64_t m, n, nnz;
+    const int64_t *row_ptr;
+    const int32_t *col_idx;
+    const float *val;
+} mps_csr64;
+
+mps_status mps_plan64(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
+                      int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out);
+mps_status mps_partition64(const int64_t *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
+                           int64_t diag_end, int64_t num_parts, int64_t items_per_part,
+                           int32_t *coord_x, int64_t *coord_y, void *stream);
+mps_status mps_spmm64_workspace_bytes(const mps_csr64 *A, int32_t K, int32_t b_dtype,
+                                      int64_t num_parts, int32_t fixup, size_t *bytes);
+mps_status mps_spmm64(const mps_csr64 *A, const void *B, int32_t b_dtype, int64_t ldb,
+                      int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                      const int64_t *coord_y, int64_t num_parts, int32_t fixup,
+                      int32_t epilogue, void *workspace, size_t workspace_bytes, void *stream);
+mps_status mps_spmm64_online_workspace_bytes(const mps_csr64 *A, int32_t K, int32_t b_dtype,
+                                             int64_t items_per_part, int64_t min_parts,
+                                             int32_t fixup, size_t *bytes);
+mps_status mps_spmm64_online(const mps_csr64 *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                             int64_t min_parts, int32_t fixup, int32_t epilogue,
+                             void *workspace, size_t workspace_bytes, void *stream);
+mps_status mps_write_stats64(const mps_csr64 *A, const int32_t *coord_x, const int64_t *coord_y,
+                             int64_t num_parts, int64_t *counts_out, void *stream);
+mps_status mps_validate_csr64(const mps_csr64 *A, int64_t *first_bad_host, void *stream);
+
 /* Debug-only validation of CSR content on the device (synchronises).  Checks
  * row_ptr[0] == 0, row_ptr non-decreasing, row_ptr[m] == nnz, 0 <= col < n.
  * *first_bad_host = -1 if valid, else the first offending row_ptr index (< m+1) or

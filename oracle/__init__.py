@@ -51,6 +51,8 @@ def _L():
         lib.oracle_plan.argtypes = [_i64, _i64, _i64, _i64, _p, _p]
         lib.oracle_merge_coord.argtypes = [_p, _i64, _i64, _i64, _p, _p]
         lib.oracle_partition.argtypes = [_p, _i64, _i64, _i64, _i64, _i64, _i64, _p, _p]
+        lib.oracle_merge_coord64.argtypes = [_p, _i64, _i64, _i64, _p, _p]
+        lib.oracle_partition64.argtypes = [_p, _i64, _i64, _i64, _i64, _i64, _i64, _p, _p]
         lib.oracle_merge_walk.argtypes = [_p, _i64, _i64, _p, _p]
         lib.oracle_alg2_emulate.argtypes = [_i64, _p, _p, _p, _p, _i64, _i32, _p, _p, _i64,
                                             _p, _i64, _p, _p]
@@ -134,6 +136,20 @@ def partition(row_ptr, num_parts, items_per_part, diag_begin=0, diag_end=None):
     cy = np.zeros(num_parts + 1, np.int32)
     rc = _L().oracle_partition(_ptr(rp), m, nnz, diag_begin, diag_end, num_parts,
                                items_per_part, _ptr(cx), _ptr(cy))
+    if rc != 0:
+        raise ValueError("invalid partition arguments")
+    return cx, cy
+
+
+def partition64(row_ptr, num_parts, items_per_part, diag_begin=0, diag_end=None):
+    """O4c with int64 row offsets (NEXT-4): (cx int32[P+1], cy int64[P+1])."""
+    rp = _c(row_ptr, np.int64)
+    m, nnz = rp.shape[0] - 1, int(rp[-1])
+    diag_end = m + nnz if diag_end is None else diag_end
+    cx = np.zeros(num_parts + 1, np.int32)
+    cy = np.zeros(num_parts + 1, np.int64)
+    rc = _L().oracle_partition64(_ptr(rp), m, nnz, diag_begin, diag_end, num_parts,
+                                 items_per_part, _ptr(cx), _ptr(cy))
     if rc != 0:
         raise ValueError("invalid partition arguments")
     return cx, cy

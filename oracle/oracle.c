@@ -20,6 +20,7 @@
  *   O2 (same call)           Bnd = |A|*|B|, used by the tolerance    (north star)
  *   O3 oracle_dense_spmm_f64 dense brute force                       (textbook)
  *   O4 oracle_plan / oracle_merge_coord / oracle_partition           (Alg. 1)
+ *      oracle_merge_coord64 / oracle_partition64: the same, int64 RP  (NEXT-4)
  *   O5 oracle_merge_walk     explicit merge of row ends and nnz      (Fig. 3 text)
  *   O6 oracle_alg2_emulate   serial Alg. 2 with write counters       (Alg. 2)
  *   O7 oracle_shard          merge-path shard bounds + tail rows     (north star stage 4)
@@ -173,6 +174,41 @@ int oracle_partition(const int32_t *RP, int64_t m, int64_t nnz, int64_t diag_beg
         oracle_merge_coord(RP, m, nnz, diag_begin + off, &x, &y);
         cx[p] = (int32_t)x;
         cy[p] = (int32_t)y;
+    }
+    return 0;
+}
+
+/* O4 with 64-bit row offsets (NEXT-4: graphs with m + nnz >= 2^31).  The same */
+/* closed form as oracle_merge_coord / oracle_partition, on int64 RP; rows     */
+/* stay < 2^31 so x is returned as int32, y as int64.                          */
+int oracle_merge_coord64(const int64_t *RP, int64_t m, int64_t nnz, int64_t d,
+                         int64_t *x_out, int64_t *y_out)
+{
+    if (d < 0 || d > m + nnz) return 1;
+    int64_t lo = d - nnz > 0 ? d - nnz : 0;
+    int64_t hi = d < m ? d : m;
+    while (lo < hi) {
+        int64_t mid = lo + (hi - lo + 1) / 2;
+        if (mid + RP[mid] <= d) lo = mid;
+        else hi = mid - 1;
+    }
+    *x_out = lo;
+    *y_out = d - lo;
+    return 0;
+}
+
+int oracle_partition64(const int64_t *RP, int64_t m, int64_t nnz, int64_t diag_begin,
+                       int64_t diag_end, int64_t P, int64_t L, int32_t *cx, int64_t *cy)
+{
+    if (P < 1 || L < 0 || diag_begin < 0 || diag_end < diag_begin || diag_end > m + nnz)
+        return 1;
+    for (int64_t p = 0; p <= P; ++p) {
+        int64_t off = p * L;
+        if (off > diag_end - diag_begin) off = diag_end - diag_begin;
+        int64_t x, y;
+        oracle_merge_coord64(RP, m, nnz, diag_begin + off, &x, &y);
+        cx[p] = (int32_t)x;
+        cy[p] = y;
     }
     return 0;
 }

@@ -24,6 +24,12 @@ class mps_csr(ctypes.Structure):
                 ("val", _p)]
 
 
+class mps_csr64(ctypes.Structure):
+    """NEXT-4: int64 row_ptr (m + nnz >= 2^31); col_idx stays int32."""
+    _fields_ = [("m", _i64), ("n", _i64), ("nnz", _i64), ("row_ptr", _p), ("col_idx", _p),
+                ("val", _p)]
+
+
 class MpsError(RuntimeError):
     def __init__(self, status, fn, detail):
         super().__init__("%s -> %s: %s" % (fn, _STATUS.get(status, status), detail))
@@ -65,6 +71,15 @@ _SIGS = {
                        _p, _i32, _p, _sz, _p],
     "mps_apply_tails": [_p, _p, _p, _i32, _i32, _i32, _p, _i64, _p],
     "mps_validate_csr": [_p, _p, _p],
+    "mps_plan64": [_i64, _i64, _i32, _i32, _i64, _i64, _p, _p],
+    "mps_partition64": [_p, _i64, _i64, _i64, _i64, _i64, _i64, _p, _p, _p],
+    "mps_spmm64_workspace_bytes": [_p, _i32, _i32, _i64, _i32, _p],
+    "mps_spmm64": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _i32, _p, _sz, _p],
+    "mps_spmm64_online_workspace_bytes": [_p, _i32, _i32, _i64, _i64, _i32, _p],
+    "mps_spmm64_online": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _i32, _p, _sz,
+                          _p],
+    "mps_write_stats64": [_p, _p, _p, _i64, _p, _p],
+    "mps_validate_csr64": [_p, _p, _p],
 }
 _RESTYPES = {"mps_abi_version": ctypes.c_int, "mps_status_string": ctypes.c_char_p,
              "mps_last_error": ctypes.c_char_p}

@@ -44,15 +44,19 @@ def _fix(f):
 
 
 class CSR:
-    """A (m x n) in CSR on one device: int32 row_ptr[m+1], int32 col_idx[nnz], fp32 val."""
+    """A (m x n) in CSR on one device: row_ptr[m+1], int32 col_idx[nnz], fp32 val.
+
+    row_ptr int32 uses the int32 entry points (m + nnz < 2^31); row_ptr int64 uses the
+    NEXT-4 64-bit ones (mps_csr64: nnz up to 2^62, m and n < 2^31)."""
 
     def __init__(self, row_ptr, col_idx, val, n_cols):
         self.row_ptr, self.col_idx, self.val = row_ptr, col_idx, val
         self.m = int(row_ptr.numel()) - 1
         self.n = int(n_cols)
         self.nnz = int(col_idx.numel())
-        assert row_ptr.dtype == torch.int32 and col_idx.dtype == torch.int32
+        assert row_ptr.dtype in (torch.int32, torch.int64) and col_idx.dtype == torch.int32
         assert val.dtype == torch.float32 and val.numel() == self.nnz
+        self.wide = row_ptr.dtype == torch.int64
 
     @classmethod
     def from_numpy(cls, row_ptr, col_idx, val, n_cols, device="cuda"):
@@ -63,9 +67,9 @@ class CSR:
     def device(self):
         return self.row_ptr.device
 
-    def struct(self) -> L.mps_csr:
-        return L.mps_csr(self.m, self.n, self.nnz, _p(self.row_ptr), _p(self.col_idx),
-                         _p(self.val))
+    def struct(self):
+        cls = L.mps_csr64 if self.wide else L.mps_csr
+        return cls(self.m, self.n, self.nnz, _p(self.row_ptr), _p(self.col_idx), _p(self.val))
 
 
 def mps_csr_host(row_ptr, col_idx, val, n_cols) -> L.mps_csr:
@@ -75,10 +79,12 @@ def mps_csr_host(row_ptr, col_idx, val, n_cols) -> L.mps_csr:
     return L.mps_csr(m, n_cols, nnz, _p(row_ptr), _p(col_idx), _p(val))
 
 
-def plan(m, nnz, K, b_dtype=L.MPS_DT_F32, items_per_part=0, min_parts=0):
-    """a1: (P, L) = merge-path thread count and items per thread (Alg. 1 l.2-3)."""
+def plan(m, nnz, K, b_dtype=L.MPS_DT_F32, items_per_part=0, min_parts=0, wide=False):
+    """a1: (P, L) = merge-path thread count and items per thread (Alg. 1 l.2-3).
+    wide=True: mps_plan64 (no 2^31 limit on m + nnz)."""
     P, Lp = ctypes.c_int64(), ctypes.c_int64()
-    L.mps_plan(m, nnz, K, b_dtype, items_per_part, min_parts, ctypes.byref(P), ctypes.byref(Lp))
+    f = L.mps_plan64 if wide else L.mps_plan
+    f(m, nnz, K, b_dtype, items_per_part, min_parts, ctypes.byref(P), ctypes.byref(Lp))
     return P.value, Lp.value
 
 
@@ -86,9 +92,10 @@ def partition(A: CSR, num_parts, items_per_part, diag_begin=0, diag_end=None, st
     """a2: coordinates (x_p, y_p), p = 0..P, of the merge-path diagonals (Alg. 1 l.4-7)."""
     diag_end = A.m + A.nnz if diag_end is None else diag_end
     cx = torch.empty(num_parts + 1, dtype=torch.int32, device=A.device)
-    cy = torch.empty(num_parts + 1, dtype=torch.int32, device=A.device)
-    L.mps_partition(_p(A.row_ptr), A.m, A.nnz, diag_begin, diag_end, num_parts, items_per_part,
-                    _p(cx), _p(cy), _stream(stream))
+    cy = torch.empty(num_parts + 1, dtype=A.row_ptr.dtype, device=A.device)
+    f = L.mps_partition64 if A.wide else L.mps_partition
+    f(_p(A.row_ptr), A.m, A.nnz, diag_begin, diag_end, num_parts, items_per_part,
+      _p(cx), _p(cy), _stream(stream))
     return cx, cy
 
 
@@ -103,7 +110,7 @@ class Schedule:
     @classmethod
     def build(cls, A: CSR, K, b_dtype=torch.float32, items_per_part=0, min_parts=0, stream=None):
         dt = L.MPS_DT_BF16 if b_dtype == torch.bfloat16 else L.MPS_DT_F32
-        P, Lp = plan(A.m, A.nnz, K, dt, items_per_part, min_parts)
+        P, Lp = plan(A.m, A.nnz, K, dt, items_per_part, min_parts, wide=A.wide)
         cx, cy = partition(A, P, Lp, stream=stream)
         return cls(P, Lp, cx, cy)
 
@@ -131,7 +138,22 @@ def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomi
     a = A.struct()
     nb = ctypes.c_size_t()
     st = _stream(stream)
-    if schedule is not None:
+    if A.wide:      # NEXT-4: 64-bit non-zero indices
+        if schedule is not None:
+            L.mps_spmm64_workspace_bytes(ctypes.byref(a), K, dt, schedule.num_parts,
+                                         _fix(fixup), ctypes.byref(nb))
+            ws = _ws(nb.value, A.device)
+            L.mps_spmm64(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
+                         _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts,
+                         _fix(fixup), EPILOGUE[epilogue], _p(ws), nb.value, st)
+        else:
+            L.mps_spmm64_online_workspace_bytes(ctypes.byref(a), K, dt, items_per_part,
+                                                min_parts, _fix(fixup), ctypes.byref(nb))
+            ws = _ws(nb.value, A.device)
+            L.mps_spmm64_online(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
+                                items_per_part, min_parts, _fix(fixup), EPILOGUE[epilogue],
+                                _p(ws), nb.value, st)
+    elif schedule is not None:
         L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt, schedule.num_parts, _fix(fixup),
                                    ctypes.byref(nb))
         ws = _ws(nb.value, A.device)
@@ -236,7 +258,7 @@ def write_stats(A: CSR, schedule: Schedule, stream=None):
     """Fig. 5 statistic: (#atomic row updates, #regular row stores) under Alg. 2."""
     cnt = torch.empty(2, dtype=torch.int64, device=A.device)
     a = A.struct()
-    L.mps_write_stats(ctypes.byref(a), _p(schedule.coord_x), _p(schedule.coord_y),
+    (L.mps_write_stats64 if A.wide else L.mps_write_stats)(ctypes.byref(a), _p(schedule.coord_x), _p(schedule.coord_y),
                       schedule.num_parts, _p(cnt), _stream(stream))
     c = cnt.cpu()
     return int(c[0]), int(c[1])
@@ -246,5 +268,5 @@ def validate_csr(A: CSR, stream=None) -> int:
     """-1 if A's CSR content is valid, else the first offending index (synchronises)."""
     a = A.struct()
     bad = ctypes.c_int64()
-    L.mps_validate_csr(ctypes.byref(a), ctypes.byref(bad), _stream(stream))
+    (L.mps_validate_csr64 if A.wide else L.mps_validate_csr)(ctypes.byref(a), ctypes.byref(bad), _stream(stream))
     return bad.value

@@ -4,6 +4,7 @@
 #include <cstring>
 #include <cstdarg>
 #include <cstdlib>
+#include <type_traits>
 #include <vector>
 
 #include "mps_internal.cuh"
@@ -140,20 +141,31 @@ void tile_geometry(int32_t kt, int W, int *V, int *NR) {
     }
 }
 
-mps_status check_csr(const mps_csr *A, bool device_ptrs_needed = true) {
+// Index type of a CSR struct: int32_t (mps_csr) or int64_t (mps_csr64, NEXT-4).
+template <typename CSR>
+using idx_t = std::remove_const_t<std::remove_pointer_t<decltype(CSR::row_ptr)>>;
+
+constexpr int64_t kMaxIndex64 = (int64_t)1 << 62;
+
+template <typename CSR>
+mps_status check_csr(const CSR *A, bool device_ptrs_needed = true) {
     if (!A) return fail(MPS_ERR_INVALID, "A is NULL");
     if (A->m < 0 || A->n < 0 || A->nnz < 0) return fail(MPS_ERR_INVALID, "negative CSR size");
-    if (A->m + A->nnz >= kMaxIndex || A->n >= kMaxIndex)
-        return fail(MPS_ERR_UNSUPPORTED, "m + nnz = %lld >= 2^31 (int32 indices)",
+    if (sizeof(*A->row_ptr) == 4 && (A->m + A->nnz >= kMaxIndex || A->n >= kMaxIndex))
+        return fail(MPS_ERR_UNSUPPORTED, "m + nnz = %lld >= 2^31 (int32 indices; use mps_csr64)",
                     (long long)(A->m + A->nnz));
+    if (sizeof(*A->row_ptr) == 8 &&
+        (A->m >= kMaxIndex || A->n >= kMaxIndex || A->nnz >= kMaxIndex64))
+        return fail(MPS_ERR_UNSUPPORTED, "mps_csr64 needs m, n < 2^31 and nnz < 2^62");
     if (device_ptrs_needed && A->m > 0 && !A->row_ptr) return fail(MPS_ERR_INVALID, "row_ptr NULL");
     if (device_ptrs_needed && A->nnz > 0 && (!A->col_idx || !A->val))
         return fail(MPS_ERR_INVALID, "col_idx/val NULL");
     return MPS_OK;
 }
 
+template <typename CSR>
 mps_status check_dense(const void *B, int32_t dt, int64_t ldb, int32_t K, const float *C,
-                       int64_t ldc, const mps_csr *A) {
+                       int64_t ldc, const CSR *A) {
     if (dt != MPS_DT_F32 && dt != MPS_DT_BF16) return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", dt);
     if (K < 0) return fail(MPS_ERR_INVALID, "K < 0");
     if (K > 0 && (ldb < K || ldc < K)) return fail(MPS_ERR_INVALID, "ldb/ldc < K");
@@ -174,7 +186,8 @@ size_t carry_bytes(int64_t P, int32_t K, const Vec &v) {
 int resolve_fix(int32_t fixup) { return fixup == MPS_FIXUP_CARRY ? mps::FIX_CARRY : mps::FIX_ATOMIC; }
 
 // host coordinate of diagonal d (shard bounds): x = max{x : x + rp[x] <= d}
-int64_t host_diag_x(const int32_t *rp, int64_t m, int64_t nnz, int64_t d) {
+template <typename IT>
+int64_t host_diag_x(const IT *rp, int64_t m, int64_t nnz, int64_t d) {
     int64_t lo = (d > nnz ? d - nnz : 0) + 1, hi = (d < m ? d : m) + 1;
     while (lo < hi) {
         int64_t mid = (lo + hi) >> 1;
@@ -185,11 +198,12 @@ int64_t host_diag_x(const int32_t *rp, int64_t m, int64_t nnz, int64_t d) {
 }
 
 // Run a3 (+ a4 carry reduction) over all column tiles for a ready schedule.
-mps_status run_segments(mps::SegArgs base, int32_t dt, int32_t K, const Vec &v, int fix,
+template <typename IT>
+mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec &v, int fix,
                         void *workspace, cudaStream_t s) {
     const int eb = elt_bytes(dt);
     for (int32_t c0 = 0; c0 < K; c0 += v.tile) {
-        mps::SegArgs a = base;
+        mps::SegArgsT<IT> a = base;
         const int32_t kt = (K - c0) < v.tile ? (K - c0) : v.tile;
         a.K = kt;
         a.B = (const char *)base.B + (size_t)c0 * eb;
@@ -248,14 +262,19 @@ const char *mps_status_string(mps_status s) {
 
 const char *mps_last_error(void) { return g_err; }
 
-mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
-                    int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out) {
+}  // extern "C"
+
+static mps_status plan_impl(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype,
+                            int64_t items_per_part, int64_t min_parts, int64_t *num_parts_out,
+                            int64_t *items_per_part_out, bool wide) {
     if (m < 0 || nnz < 0 || K < 0 || items_per_part < 0 || min_parts < 0)
         return fail(MPS_ERR_INVALID, "negative plan argument");
     if (!num_parts_out || !items_per_part_out) return fail(MPS_ERR_INVALID, "NULL output");
     if (b_dtype != MPS_DT_F32 && b_dtype != MPS_DT_BF16)
         return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", b_dtype);
-    if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (!wide && m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (wide && (m >= kMaxIndex || nnz >= kMaxIndex64))
+        return fail(MPS_ERR_UNSUPPORTED, "m >= 2^31 or nnz >= 2^62");
     const int64_t cost = items_per_part ? items_per_part : default_cost(m, nnz, K, b_dtype);
     const int64_t pmin = min_parts ? min_parts : kDefaultMinParts;
     const int64_t M = m + nnz;                      // Alg. 1 line 2
@@ -266,20 +285,52 @@ mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t 
     return MPS_OK;
 }
 
-mps_status mps_partition(const int32_t *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
-                         int64_t diag_end, int64_t num_parts, int64_t items_per_part,
-                         int32_t *coord_x, int32_t *coord_y, void *stream) {
+template <typename IT>
+static mps_status partition_impl(const IT *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
+                                 int64_t diag_end, int64_t num_parts, int64_t items_per_part,
+                                 int32_t *coord_x, IT *coord_y, void *stream) {
     if (m < 0 || nnz < 0 || num_parts < 1 || items_per_part < 0)
         return fail(MPS_ERR_INVALID, "bad partition sizes");
-    if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (sizeof(IT) == 4 && m + nnz >= kMaxIndex)
+        return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (sizeof(IT) == 8 && (m >= kMaxIndex || nnz >= kMaxIndex64))
+        return fail(MPS_ERR_UNSUPPORTED, "m >= 2^31 or nnz >= 2^62");
     if (diag_begin < 0 || diag_end < diag_begin || diag_end > m + nnz)
         return fail(MPS_ERR_INVALID, "diagonal range outside [0, m + nnz]");
     if (!row_ptr || !coord_x || !coord_y) return fail(MPS_ERR_INVALID, "NULL pointer");
-    MPS_CUDA(mps::launch_partition(row_ptr, m, nnz, diag_begin, diag_end - diag_begin, num_parts,
-                                   items_per_part, coord_x, coord_y, nullptr, 0, 0, 0, -1,
-                                   nullptr, (cudaStream_t)stream),
+    MPS_CUDA(mps::launch_partition<IT>(row_ptr, m, nnz, diag_begin, diag_end - diag_begin,
+                                       num_parts, items_per_part, coord_x, coord_y, nullptr, 0, 0,
+                                       0, -1, nullptr, (cudaStream_t)stream),
              "partition kernel");
     return MPS_OK;
+}
+
+extern "C" {
+
+mps_status mps_plan(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
+                    int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out) {
+    return plan_impl(m, nnz, K, b_dtype, items_per_part, min_parts, num_parts_out,
+                     items_per_part_out, false);
+}
+
+mps_status mps_plan64(int64_t m, int64_t nnz, int32_t K, int32_t b_dtype, int64_t items_per_part,
+                      int64_t min_parts, int64_t *num_parts_out, int64_t *items_per_part_out) {
+    return plan_impl(m, nnz, K, b_dtype, items_per_part, min_parts, num_parts_out,
+                     items_per_part_out, true);
+}
+
+mps_status mps_partition64(const int64_t *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
+                           int64_t diag_end, int64_t num_parts, int64_t items_per_part,
+                           int32_t *coord_x, int64_t *coord_y, void *stream) {
+    return partition_impl<int64_t>(row_ptr, m, nnz, diag_begin, diag_end, num_parts,
+                                   items_per_part, coord_x, coord_y, stream);
+}
+
+mps_status mps_partition(const int32_t *row_ptr, int64_t m, int64_t nnz, int64_t diag_begin,
+                         int64_t diag_end, int64_t num_parts, int64_t items_per_part,
+                         int32_t *coord_x, int32_t *coord_y, void *stream) {
+    return partition_impl<int32_t>(row_ptr, m, nnz, diag_begin, diag_end, num_parts,
+                                   items_per_part, coord_x, coord_y, stream);
 }
 
 mps_status mps_partition_split(const int32_t *row_ptr, int64_t m, int64_t nnz,
@@ -298,8 +349,17 @@ mps_status mps_partition_split(const int32_t *row_ptr, int64_t m, int64_t nnz,
     return MPS_OK;
 }
 
-mps_status mps_spmm_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
-                                    int64_t num_parts, int32_t fixup, size_t *bytes) {
+}  // extern "C"
+
+// ---------------------------------------------------------------------------------
+// a3 + a4 implementations shared by the int32 (mps_csr) and int64 (mps_csr64, NEXT-4)
+// entry points.  CSR is the public struct; its row_ptr type is the index type IT.
+// ---------------------------------------------------------------------------------
+namespace {
+
+template <typename CSR>
+mps_status spmm_ws_impl(const CSR *A, int32_t K, int32_t b_dtype, int64_t num_parts,
+                        int32_t fixup, size_t *bytes) {
     mps_status st = check_csr(A, false);
     if (st) return st;
     if (!bytes || num_parts < 1 || K < 0) return fail(MPS_ERR_INVALID, "bad arguments");
@@ -318,9 +378,9 @@ mps_status mps_spmm_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype
     return MPS_OK;
 }
 
-mps_status mps_zero_split_rows(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
-                               int64_t num_parts, float *C, int64_t ldc, int32_t K,
-                               void *stream) {
+template <typename CSR>
+mps_status zero_split_impl(const CSR *A, const int32_t *coord_x, const idx_t<CSR> *coord_y,
+                           int64_t num_parts, float *C, int64_t ldc, int32_t K, void *stream) {
     mps_status st = check_csr(A);
     if (st) return st;
     if (num_parts < 1 || K < 0 || (K > 0 && ldc < K)) return fail(MPS_ERR_INVALID, "bad arguments");
@@ -332,72 +392,12 @@ mps_status mps_zero_split_rows(const mps_csr *A, const int32_t *coord_x, const i
     return MPS_OK;
 }
 
-mps_status mps_spmm(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
-                    float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
-                    int64_t num_parts, int32_t fixup, void *workspace, size_t workspace_bytes,
-                    void *stream) {
-    if (resolve_fix(fixup) == mps::FIX_ATOMIC) {
-        mps_status st = check_csr(A);
-        if (st) return st;
-        if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
-        if (num_parts < 1) return fail(MPS_ERR_INVALID, "num_parts < 1");
-        if (K == 0 || A->m == 0) return MPS_OK;
-        if ((st = mps_zero_split_rows(A, coord_x, coord_y, num_parts, C, ldc, K, stream)))
-            return st;
-    }
-    return mps_spmm_segments(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
-                             workspace, workspace_bytes, stream);
-}
-
-mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                             int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
-                             const int32_t *coord_y, int64_t num_parts, int32_t fixup,
-                             void *workspace, size_t workspace_bytes, void *stream) {
-    return mps_spmm_segments_hot(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts,
-                                 fixup, nullptr, workspace, workspace_bytes, stream);
-}
-
-static mps_status segments_impl(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                                int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
-                                const int32_t *coord_y, int64_t num_parts, int32_t fixup,
-                                const uint32_t *hot_bitmap, int32_t relu, void *workspace,
-                                size_t workspace_bytes, void *stream);
-
-mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                                 int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
-                                 const int32_t *coord_y, int64_t num_parts, int32_t fixup,
-                                 const uint32_t *hot_bitmap, void *workspace,
-                                 size_t workspace_bytes, void *stream) {
-    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
-                         hot_bitmap, 0, workspace, workspace_bytes, stream);
-}
-
-mps_status mps_spmm_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
-                       float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
-                       int64_t num_parts, int32_t fixup, int32_t epilogue,
-                       const uint32_t *hot_bitmap, void *workspace, size_t workspace_bytes,
-                       void *stream) {
-    if (epilogue != MPS_EPI_NONE && epilogue != MPS_EPI_RELU)
-        return fail(MPS_ERR_UNSUPPORTED, "epilogue %d", epilogue);
-    if (resolve_fix(fixup) == mps::FIX_ATOMIC) {
-        mps_status st = check_csr(A);
-        if (st) return st;
-        if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
-        if (num_parts < 1) return fail(MPS_ERR_INVALID, "num_parts < 1");
-        if (K == 0 || A->m == 0) return MPS_OK;
-        if ((st = mps_zero_split_rows(A, coord_x, coord_y, num_parts, C, ldc, K, stream)))
-            return st;
-    }
-    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
-                         hot_bitmap, epilogue == MPS_EPI_RELU, workspace, workspace_bytes,
-                         stream);
-}
-
-static mps_status segments_impl(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                                int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
-                                const int32_t *coord_y, int64_t num_parts, int32_t fixup,
-                                const uint32_t *hot_bitmap, int32_t relu, void *workspace,
-                                size_t workspace_bytes, void *stream) {
+template <typename CSR>
+mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                         float *C, int64_t ldc, const int32_t *coord_x,
+                         const idx_t<CSR> *coord_y, int64_t num_parts, int32_t fixup,
+                         const uint32_t *hot_bitmap, int32_t relu, void *workspace,
+                         size_t workspace_bytes, void *stream) {
     mps_status st = check_csr(A);
     if (st) return st;
     if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
@@ -410,8 +410,7 @@ static mps_status segments_impl(const mps_csr *A, const void *B, int32_t b_dtype
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes,
                     carry_bytes(num_parts, K, v));
     if (fix == mps::FIX_CARRY && !workspace) return fail(MPS_ERR_WORKSPACE, "workspace NULL");
-    cudaStream_t s = (cudaStream_t)stream;
-    mps::SegArgs a{};
+    mps::SegArgsT<idx_t<CSR>> a{};
     a.rp = A->row_ptr;
     a.col = A->col_idx;
     a.val = A->val;
@@ -429,22 +428,39 @@ static mps_status segments_impl(const mps_csr *A, const void *B, int32_t b_dtype
     a.nnz_end = A->nnz;
     a.hot = hot_bitmap;
     a.relu = relu;
-    return run_segments(a, b_dtype, K, v, fix, workspace, s);
+    return run_segments(a, b_dtype, K, v, fix, workspace, (cudaStream_t)stream);
 }
 
-static size_t hot_scratch_bytes(int64_t n) {
+template <typename CSR>
+mps_status spmm_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                        float *C, int64_t ldc, const int32_t *coord_x,
+                        const idx_t<CSR> *coord_y, int64_t num_parts, int32_t fixup,
+                        int32_t epilogue, const uint32_t *hot_bitmap, void *workspace,
+                        size_t workspace_bytes, void *stream) {
+    if (epilogue != MPS_EPI_NONE && epilogue != MPS_EPI_RELU)
+        return fail(MPS_ERR_UNSUPPORTED, "epilogue %d", epilogue);
+    if (resolve_fix(fixup) == mps::FIX_ATOMIC) {
+        mps_status st = check_csr(A);
+        if (st) return st;
+        if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
+        if (num_parts < 1) return fail(MPS_ERR_INVALID, "num_parts < 1");
+        if (K == 0 || A->m == 0) return MPS_OK;
+        if ((st = zero_split_impl(A, coord_x, coord_y, num_parts, C, ldc, K, stream)))
+            return st;
+    }
+    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                         hot_bitmap, epilogue == MPS_EPI_RELU, workspace, workspace_bytes,
+                         stream);
+}
+
+size_t hot_scratch_bytes(int64_t n) {
     return align_up((size_t)n * 4, 256) + align_up(34 * 4, 256);
 }
-static size_t hot_bitmap_bytes(int64_t n) { return align_up((size_t)((n + 31) / 32) * 4, 256); }
+size_t hot_bitmap_bytes(int64_t n) { return align_up((size_t)((n + 31) / 32) * 4, 256); }
 
-mps_status mps_hot_rows_workspace_bytes(int64_t n, size_t *bytes) {
-    if (n < 0 || !bytes) return fail(MPS_ERR_INVALID, "bad arguments");
-    *bytes = hot_scratch_bytes(n);
-    return MPS_OK;
-}
-
-mps_status mps_hot_rows(const mps_csr *A, int64_t budget_rows, uint32_t *hot_bitmap,
-                        void *workspace, size_t workspace_bytes, void *stream) {
+template <typename CSR>
+mps_status hot_rows_impl(const CSR *A, int64_t budget_rows, uint32_t *hot_bitmap,
+                         void *workspace, size_t workspace_bytes, void *stream) {
     mps_status st = check_csr(A);
     if (st) return st;
     if (budget_rows < 0 || (A->n > 0 && !hot_bitmap)) return fail(MPS_ERR_INVALID, "bad arguments");
@@ -461,13 +477,9 @@ mps_status mps_hot_rows(const mps_csr *A, int64_t budget_rows, uint32_t *hot_bit
 }
 
 // Use degree-aware L2 residency when the gathered B is larger than half the L2.
-static int64_t hot_budget_rows(const mps_csr *A, int32_t K, int32_t dt) {
-    int dev = 0, l2 = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess ||
-        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev) != cudaSuccess || l2 <= 0)
-        l2 = 126 << 20;
+int64_t hot_budget_rows(int64_t n, int32_t K, int32_t dt) {
     const double row = (double)K * elt_bytes(dt);
-    if ((double)A->n * row <= 0.5 * (double)l2) return -1;     // B fits: plain evict_last
+    if ((double)n * row <= 0.5 * (double)l2_bytes()) return -1;     // B fits: plain evict_last
     // Off by default: measured on B200 (profiles/r01/hot_rows.md) the static hub policy
     // gains <= 5% in the segment kernel and its per-call pre-pass costs more online.
     static const double frac = [] {
@@ -475,58 +487,46 @@ static int64_t hot_budget_rows(const mps_csr *A, int32_t K, int32_t dt) {
         return e ? atof(e) : 0.0;
     }();
     if (frac <= 0) return -1;
-    return (int64_t)(frac * (double)l2 / row);
+    return (int64_t)(frac * (double)l2_bytes() / row);
 }
 
-mps_status mps_hot_budget_rows(const mps_csr *A, int32_t K, int32_t b_dtype,
-                               int64_t *budget_rows_out) {
-    mps_status st = check_csr(A, false);
-    if (st) return st;
-    if (!budget_rows_out || K < 0) return fail(MPS_ERR_INVALID, "bad arguments");
-    if (b_dtype != MPS_DT_F32 && b_dtype != MPS_DT_BF16)
-        return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", b_dtype);
-    *budget_rows_out = K > 0 ? hot_budget_rows(A, K, b_dtype) : -1;
-    return MPS_OK;
-}
-
-static size_t online_bytes(int64_t P, int32_t K, const Vec &v, int fix, int64_t n = 0) {
-    size_t b = align_up((size_t)(P + 1) * 4, 256) * 2;
+// online workspace: coord_x int32[P+1], coord_y IT[P+1], carry records, hot-row scratch
+size_t online_bytes(int64_t P, int32_t K, const Vec &v, int fix, int64_t n = 0,
+                    size_t ysize = 4) {
+    size_t b = align_up((size_t)(P + 1) * 4, 256) + align_up((size_t)(P + 1) * ysize, 256);
     if (fix == mps::FIX_CARRY) b += carry_bytes(P, K, v);
     if (n > 0) b += hot_bitmap_bytes(n) + hot_scratch_bytes(n);
     return b;
 }
 
-mps_status mps_spmm_online_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
-                                           int64_t items_per_part, int64_t min_parts,
-                                           int32_t fixup, size_t *bytes) {
+template <typename CSR>
+mps_status online_ws_impl(const CSR *A, int32_t K, int32_t b_dtype, int64_t items_per_part,
+                          int64_t min_parts, int32_t fixup, size_t *bytes) {
     mps_status st = check_csr(A, false);
     if (st) return st;
     if (!bytes) return fail(MPS_ERR_INVALID, "bytes NULL");
     int64_t P, L;
-    if ((st = mps_plan(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
+    if ((st = plan_impl(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L,
+                        sizeof(idx_t<CSR>) == 8)))
+        return st;
     Vec vmin;
     vmin.W = 1;
     vmin.tile = 128;
     const Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
     const int fix = resolve_fix(fixup);
-    const int64_t nh = hot_budget_rows(A, K, b_dtype) >= 0 ? A->n : 0;
-    size_t a = online_bytes(P, K, v, fix, nh), b = online_bytes(P, K, vmin, fix, nh);
+    const int64_t nh = hot_budget_rows(A->n, K, b_dtype) >= 0 ? A->n : 0;
+    const size_t ys = sizeof(idx_t<CSR>);
+    size_t a = online_bytes(P, K, v, fix, nh, ys), b = online_bytes(P, K, vmin, fix, nh, ys);
     *bytes = a > b ? a : b;
     return MPS_OK;
 }
 
-mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                           int32_t K, float *C, int64_t ldc, int64_t items_per_part,
-                           int64_t min_parts, int32_t fixup, void *workspace,
-                           size_t workspace_bytes, void *stream) {
-    return mps_spmm_online_ex(A, B, b_dtype, ldb, K, C, ldc, items_per_part, min_parts, fixup,
-                              MPS_EPI_NONE, workspace, workspace_bytes, stream);
-}
-
-mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                              int32_t K, float *C, int64_t ldc, int64_t items_per_part,
-                              int64_t min_parts, int32_t fixup, int32_t epilogue,
-                              void *workspace, size_t workspace_bytes, void *stream) {
+template <typename CSR>
+mps_status online_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                          float *C, int64_t ldc, int64_t items_per_part, int64_t min_parts,
+                          int32_t fixup, int32_t epilogue, void *workspace,
+                          size_t workspace_bytes, void *stream) {
+    using IT = idx_t<CSR>;
     if (epilogue != MPS_EPI_NONE && epilogue != MPS_EPI_RELU)
         return fail(MPS_ERR_UNSUPPORTED, "epilogue %d", epilogue);
     mps_status st = check_csr(A);
@@ -534,31 +534,35 @@ mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, 
     if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
     if (K == 0 || A->m == 0) return MPS_OK;
     int64_t P, L;
-    if ((st = mps_plan(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L))) return st;
+    if ((st = plan_impl(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L,
+                        sizeof(IT) == 8)))
+        return st;
     const int fix = resolve_fix(fixup);
     const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n);
-    const int64_t hot_rows = hot_budget_rows(A, K, b_dtype);
+    const int64_t hot_rows = hot_budget_rows(A->n, K, b_dtype);
     const int64_t nh = hot_rows >= 0 ? A->n : 0;
-    const size_t need = online_bytes(P, K, v, fix, nh);
+    const size_t need = online_bytes(P, K, v, fix, nh, sizeof(IT));
     if (!workspace || workspace_bytes < need)
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
     cudaStream_t s = (cudaStream_t)stream;
+    const size_t xb = align_up((size_t)(P + 1) * 4, 256);
+    const size_t yb = align_up((size_t)(P + 1) * sizeof(IT), 256);
     int32_t *cx = (int32_t *)workspace;
-    int32_t *cy = (int32_t *)((char *)workspace + align_up((size_t)(P + 1) * 4, 256));
-    void *rec = (char *)workspace + align_up((size_t)(P + 1) * 4, 256) * 2;
+    IT *cy = (IT *)((char *)workspace + xb);
+    void *rec = (char *)workspace + xb + yb;
     uint32_t *bitmap = nullptr;
     if (nh > 0) {
-        char *hb = (char *)workspace + online_bytes(P, K, v, fix, 0);
+        char *hb = (char *)workspace + online_bytes(P, K, v, fix, 0, sizeof(IT));
         bitmap = (uint32_t *)hb;
-        mps_status hs = mps_hot_rows(A, hot_rows, bitmap, hb + hot_bitmap_bytes(A->n),
-                                     hot_scratch_bytes(A->n), stream);
+        mps_status hs = hot_rows_impl(A, hot_rows, bitmap, hb + hot_bitmap_bytes(A->n),
+                                      hot_scratch_bytes(A->n), stream);
         if (hs) return hs;
     }
-    MPS_CUDA(mps::launch_partition(A->row_ptr, A->m, A->nnz, 0, A->m + A->nnz, P, L, cx, cy,
-                                   fix == mps::FIX_ATOMIC ? C : nullptr, ldc, 0, K, -1, nullptr,
-                                   s),
+    MPS_CUDA(mps::launch_partition<IT>(A->row_ptr, A->m, A->nnz, 0, A->m + A->nnz, P, L, cx, cy,
+                                       fix == mps::FIX_ATOMIC ? C : nullptr, ldc, 0, K, -1,
+                                       nullptr, s),
              "partition kernel");
-    mps::SegArgs a{};
+    mps::SegArgsT<IT> a{};
     a.rp = A->row_ptr;
     a.col = A->col_idx;
     a.val = A->val;
@@ -577,6 +581,171 @@ mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, 
     a.hot = bitmap;
     a.relu = epilogue == MPS_EPI_RELU;
     return run_segments(a, b_dtype, K, v, fix, rec, s);
+}
+
+template <typename CSR>
+mps_status write_stats_impl(const CSR *A, const int32_t *coord_x, const idx_t<CSR> *coord_y,
+                            int64_t num_parts, int64_t *counts_out, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (num_parts < 1 || !coord_x || !coord_y || !counts_out)
+        return fail(MPS_ERR_INVALID, "bad arguments");
+    MPS_CUDA(mps::launch_write_stats(A->row_ptr, (int32_t)A->m, coord_x, coord_y, num_parts,
+                                     counts_out, (cudaStream_t)stream),
+             "write stats");
+    return MPS_OK;
+}
+
+template <typename CSR>
+mps_status validate_impl(const CSR *A, int64_t *first_bad_host, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (!first_bad_host) return fail(MPS_ERR_INVALID, "first_bad_host NULL");
+    *first_bad_host = -1;
+    if (A->m == 0 && A->nnz == 0) return MPS_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    unsigned long long *d = nullptr;
+    MPS_CUDA(cudaMallocAsync((void **)&d, sizeof(*d), s), "alloc");
+    const unsigned long long init = ~0ull;
+    MPS_CUDA(cudaMemcpyAsync(d, &init, sizeof(init), cudaMemcpyHostToDevice, s), "H2D");
+    MPS_CUDA(mps::launch_validate(A->row_ptr, A->col_idx, A->m, A->n, A->nnz, d, s), "validate");
+    unsigned long long h = 0;
+    MPS_CUDA(cudaMemcpyAsync(&h, d, sizeof(h), cudaMemcpyDeviceToHost, s), "D2H");
+    MPS_CUDA(cudaFreeAsync(d, s), "free");
+    MPS_CUDA(cudaStreamSynchronize(s), "sync");
+    *first_bad_host = (h == ~0ull) ? -1 : (int64_t)h;
+    return MPS_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+// ---- int32 entry points (mps_csr) ----------------------------------------------------
+mps_status mps_spmm_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                    int64_t num_parts, int32_t fixup, size_t *bytes) {
+    return spmm_ws_impl(A, K, b_dtype, num_parts, fixup, bytes);
+}
+
+mps_status mps_zero_split_rows(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
+                               int64_t num_parts, float *C, int64_t ldc, int32_t K,
+                               void *stream) {
+    return zero_split_impl(A, coord_x, coord_y, num_parts, C, ldc, K, stream);
+}
+
+mps_status mps_spmm(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                    float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
+                    int64_t num_parts, int32_t fixup, void *workspace, size_t workspace_bytes,
+                    void *stream) {
+    return spmm_ex_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                        MPS_EPI_NONE, nullptr, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                             const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                             void *workspace, size_t workspace_bytes, void *stream) {
+    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                         nullptr, 0, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                 int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                                 const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                                 const uint32_t *hot_bitmap, void *workspace,
+                                 size_t workspace_bytes, void *stream) {
+    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                         hot_bitmap, 0, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
+                       float *C, int64_t ldc, const int32_t *coord_x, const int32_t *coord_y,
+                       int64_t num_parts, int32_t fixup, int32_t epilogue,
+                       const uint32_t *hot_bitmap, void *workspace, size_t workspace_bytes,
+                       void *stream) {
+    return spmm_ex_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                        epilogue, hot_bitmap, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_hot_rows_workspace_bytes(int64_t n, size_t *bytes) {
+    if (n < 0 || !bytes) return fail(MPS_ERR_INVALID, "bad arguments");
+    *bytes = hot_scratch_bytes(n);
+    return MPS_OK;
+}
+
+mps_status mps_hot_rows(const mps_csr *A, int64_t budget_rows, uint32_t *hot_bitmap,
+                        void *workspace, size_t workspace_bytes, void *stream) {
+    return hot_rows_impl(A, budget_rows, hot_bitmap, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_hot_budget_rows(const mps_csr *A, int32_t K, int32_t b_dtype,
+                               int64_t *budget_rows_out) {
+    mps_status st = check_csr(A, false);
+    if (st) return st;
+    if (!budget_rows_out || K < 0) return fail(MPS_ERR_INVALID, "bad arguments");
+    if (b_dtype != MPS_DT_F32 && b_dtype != MPS_DT_BF16)
+        return fail(MPS_ERR_UNSUPPORTED, "b_dtype %d", b_dtype);
+    *budget_rows_out = K > 0 ? hot_budget_rows(A->n, K, b_dtype) : -1;
+    return MPS_OK;
+}
+
+mps_status mps_spmm_online_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                           int64_t items_per_part, int64_t min_parts,
+                                           int32_t fixup, size_t *bytes) {
+    return online_ws_impl(A, K, b_dtype, items_per_part, min_parts, fixup, bytes);
+}
+
+mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                           int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                           int64_t min_parts, int32_t fixup, void *workspace,
+                           size_t workspace_bytes, void *stream) {
+    return online_ex_impl(A, B, b_dtype, ldb, K, C, ldc, items_per_part, min_parts, fixup,
+                          MPS_EPI_NONE, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                              int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                              int64_t min_parts, int32_t fixup, int32_t epilogue,
+                              void *workspace, size_t workspace_bytes, void *stream) {
+    return online_ex_impl(A, B, b_dtype, ldb, K, C, ldc, items_per_part, min_parts, fixup,
+                          epilogue, workspace, workspace_bytes, stream);
+}
+
+// ---- int64 entry points (mps_csr64, NEXT-4) ------------------------------------------
+mps_status mps_spmm64_workspace_bytes(const mps_csr64 *A, int32_t K, int32_t b_dtype,
+                                      int64_t num_parts, int32_t fixup, size_t *bytes) {
+    return spmm_ws_impl(A, K, b_dtype, num_parts, fixup, bytes);
+}
+
+mps_status mps_spmm64(const mps_csr64 *A, const void *B, int32_t b_dtype, int64_t ldb,
+                      int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                      const int64_t *coord_y, int64_t num_parts, int32_t fixup,
+                      int32_t epilogue, void *workspace, size_t workspace_bytes, void *stream) {
+    return spmm_ex_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                        epilogue, nullptr, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm64_online_workspace_bytes(const mps_csr64 *A, int32_t K, int32_t b_dtype,
+                                             int64_t items_per_part, int64_t min_parts,
+                                             int32_t fixup, size_t *bytes) {
+    return online_ws_impl(A, K, b_dtype, items_per_part, min_parts, fixup, bytes);
+}
+
+mps_status mps_spmm64_online(const mps_csr64 *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, float *C, int64_t ldc, int64_t items_per_part,
+                             int64_t min_parts, int32_t fixup, int32_t epilogue,
+                             void *workspace, size_t workspace_bytes, void *stream) {
+    return online_ex_impl(A, B, b_dtype, ldb, K, C, ldc, items_per_part, min_parts, fixup,
+                          epilogue, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_write_stats64(const mps_csr64 *A, const int32_t *coord_x, const int64_t *coord_y,
+                             int64_t num_parts, int64_t *counts_out, void *stream) {
+    return write_stats_impl(A, coord_x, coord_y, num_parts, counts_out, stream);
+}
+
+mps_status mps_validate_csr64(const mps_csr64 *A, int64_t *first_bad_host, void *stream) {
+    return validate_impl(A, first_bad_host, stream);
 }
 
 // ----------------------------------------------------------------------------------
@@ -666,14 +835,7 @@ mps_status mps_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const v
 
 mps_status mps_write_stats(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
                            int64_t num_parts, int64_t *counts_out, void *stream) {
-    mps_status st = check_csr(A);
-    if (st) return st;
-    if (num_parts < 1 || !coord_x || !coord_y || !counts_out)
-        return fail(MPS_ERR_INVALID, "bad arguments");
-    MPS_CUDA(mps::launch_write_stats(A->row_ptr, (int32_t)A->m, coord_x, coord_y, num_parts,
-                                     counts_out, (cudaStream_t)stream),
-             "write stats");
-    return MPS_OK;
+    return write_stats_impl(A, coord_x, coord_y, num_parts, counts_out, stream);
 }
 
 // ----------------------------------------------------------------------------------
@@ -816,23 +978,7 @@ mps_status mps_apply_tails(const float *tails, const int32_t *X, const int32_t *
 }
 
 mps_status mps_validate_csr(const mps_csr *A, int64_t *first_bad_host, void *stream) {
-    mps_status st = check_csr(A);
-    if (st) return st;
-    if (!first_bad_host) return fail(MPS_ERR_INVALID, "first_bad_host NULL");
-    *first_bad_host = -1;
-    if (A->m == 0 && A->nnz == 0) return MPS_OK;
-    cudaStream_t s = (cudaStream_t)stream;
-    unsigned long long *d = nullptr;
-    MPS_CUDA(cudaMallocAsync((void **)&d, sizeof(*d), s), "alloc");
-    const unsigned long long init = ~0ull;
-    MPS_CUDA(cudaMemcpyAsync(d, &init, sizeof(init), cudaMemcpyHostToDevice, s), "H2D");
-    MPS_CUDA(mps::launch_validate(A->row_ptr, A->col_idx, A->m, A->n, A->nnz, d, s), "validate");
-    unsigned long long h = 0;
-    MPS_CUDA(cudaMemcpyAsync(&h, d, sizeof(h), cudaMemcpyDeviceToHost, s), "D2H");
-    MPS_CUDA(cudaFreeAsync(d, s), "free");
-    MPS_CUDA(cudaStreamSynchronize(s), "sync");
-    *first_bad_host = (h == ~0ull) ? -1 : (int64_t)h;
-    return MPS_OK;
+    return validate_impl(A, first_bad_host, stream);
 }
 
 }  // extern "C"

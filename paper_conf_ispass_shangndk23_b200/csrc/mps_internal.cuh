@@ -19,9 +19,12 @@ enum Fix : int { FIX_ATOMIC = 1, FIX_CARRY = 2 };
 // Per-launch arguments of the segment kernel (a3 + a4).  Indices are global merge-path
 // coordinates; col/val are pre-offset so that col[j] is global nnz j (shards hold a
 // slice); C row r lives at C + (r - row_base) * ldc; the row `tail_row` (a shard's cut
-// last row) is redirected to `tail`.
-struct SegArgs {
-    const int32_t *rp;
+// last row) is redirected to `tail`.  IT is the type of row_ptr and of the nnz
+// coordinate y: int32_t (M = m + nnz < 2^31) or int64_t (NEXT-4: nnz >= 2^31; rows and
+// columns stay < 2^31, so coord_x and col_idx stay int32).
+template <typename IT>
+struct SegArgsT {
+    const IT *rp;
     const int32_t *col;
     const float *val;
     const void *B;
@@ -32,7 +35,7 @@ struct SegArgs {
     int64_t row_base;
     int32_t m;          // rows of the global A
     const int32_t *cx;
-    const int32_t *cy;
+    const IT *cy;
     int64_t P;
     int32_t tail_row;   // -1: none
     float *tail;
@@ -45,25 +48,35 @@ struct SegArgs {
     int32_t relu;        // epilogue: 1 = C = max(C, 0) (complete rows at the store; cut rows
                          // by launch_relu_split after the atomics, or in the carry reduce)
 };
+using SegArgs = SegArgsT<int32_t>;
+using SegArgs64 = SegArgsT<int64_t>;
 
-// Host launchers (defined in the .cu files).
-cudaError_t launch_partition(const int32_t *rp, int64_t m, int64_t nnz, int64_t d0,
-                             int64_t span, int64_t P, int64_t L, int32_t *cx, int32_t *cy,
+// Host launchers (defined in the .cu files).  IT = int32_t or int64_t (row_ptr and the
+// nnz coordinate y).
+template <typename IT>
+cudaError_t launch_partition(const IT *rp, int64_t m, int64_t nnz, int64_t d0,
+                             int64_t span, int64_t P, int64_t L, int32_t *cx, IT *cy,
                              float *zero_C, int64_t ldc, int64_t row_base, int32_t K,
                              int32_t tail_row, float *tail, cudaStream_t s);
-cudaError_t launch_zero_split(const int32_t *rp, int32_t m, const int32_t *cx,
-                              const int32_t *cy, int64_t P, float *C, int64_t ldc,
+template <typename IT>
+cudaError_t launch_zero_split(const IT *rp, int32_t m, const int32_t *cx,
+                              const IT *cy, int64_t P, float *C, int64_t ldc,
                               int64_t row_base, int32_t K, int32_t tail_row, float *tail,
                               cudaStream_t s);
-cudaError_t launch_segments(const SegArgs &a, int b_dtype, int W, int V, int NR, int fix,
+template <typename IT>
+cudaError_t launch_segments(const SegArgsT<IT> &a, int b_dtype, int W, int V, int NR, int fix,
                             cudaStream_t s);
-cudaError_t launch_carry_reduce(const SegArgs &a, cudaStream_t s);
-cudaError_t launch_relu_split(const SegArgs &a, cudaStream_t s);
+template <typename IT>
+cudaError_t launch_carry_reduce(const SegArgsT<IT> &a, cudaStream_t s);
+template <typename IT>
+cudaError_t launch_relu_split(const SegArgsT<IT> &a, cudaStream_t s);
 cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx, int32_t n,
                                float *row, cudaStream_t s);
-cudaError_t launch_write_stats(const int32_t *rp, int32_t m, const int32_t *cx,
-                               const int32_t *cy, int64_t P, int64_t *counts, cudaStream_t s);
-cudaError_t launch_validate(const int32_t *rp, const int32_t *col, int64_t m, int64_t n,
+template <typename IT>
+cudaError_t launch_write_stats(const IT *rp, int32_t m, const int32_t *cx,
+                               const IT *cy, int64_t P, int64_t *counts, cudaStream_t s);
+template <typename IT>
+cudaError_t launch_validate(const IT *rp, const int32_t *col, int64_t m, int64_t n,
                             int64_t nnz, unsigned long long *first_bad, cudaStream_t s);
 
 cudaError_t launch_hot_columns(const int32_t *col, int64_t nnz, int64_t n, int64_t budget_rows,

@@ -9,7 +9,8 @@ namespace mps {
 // s(x) = x + rp[x] is strictly increasing with s(0) = 0; the point is
 // x = max{x : s(x) <= d} (readings R4/R5), found here as the first x in
 // (max(0, d - nnz), min(d, m)] with s(x) > d, minus one.
-__device__ __forceinline__ int64_t diag_x(const int32_t *__restrict__ rp, int64_t m,
+template <typename IT>
+__device__ __forceinline__ int64_t diag_x(const IT *__restrict__ rp, int64_t m,
                                           int64_t nnz, int64_t d) {
     int64_t lo = (d > nnz ? d - nnz : 0) + 1;
     int64_t hi = (d < m ? d : m) + 1;
@@ -24,10 +25,11 @@ __device__ __forceinline__ int64_t diag_x(const int32_t *__restrict__ rp, int64_
 // One thread per diagonal p = 0..P.  With zero_C != nullptr (atomic fix-up, online),
 // the warp then zeroes every destination row cut by one of its 32 diagonals
 // (y_p > rp[x_p]): those rows receive only atomic partial sums (reading R10).
+template <typename IT>
 __global__ void __launch_bounds__(kBlock)
-partition_kernel(const int32_t *__restrict__ rp, int64_t m, int64_t nnz, int64_t d0,
+partition_kernel(const IT *__restrict__ rp, int64_t m, int64_t nnz, int64_t d0,
                  int64_t span, int64_t P, int64_t L, int32_t *__restrict__ cx,
-                 int32_t *__restrict__ cy, float *zero_C, int64_t ldc, int64_t row_base,
+                 IT *__restrict__ cy, float *zero_C, int64_t ldc, int64_t row_base,
                  int32_t K, int32_t tail_row, float *tail) {
     const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const bool valid = p <= P;
@@ -39,7 +41,7 @@ partition_kernel(const int32_t *__restrict__ rp, int64_t m, int64_t nnz, int64_t
         x = diag_x(rp, m, nnz, d);
         y = d - x;
         cx[p] = (int32_t)x;
-        cy[p] = (int32_t)y;
+        cy[p] = (IT)y;
     }
     if (zero_C == nullptr && tail == nullptr) return;  // uniform across the grid
     const bool inside = valid && x < m && y > (int64_t)__ldg(rp + x);
@@ -54,13 +56,14 @@ partition_kernel(const int32_t *__restrict__ rp, int64_t m, int64_t nnz, int64_t
     }
 }
 
-cudaError_t launch_partition(const int32_t *rp, int64_t m, int64_t nnz, int64_t d0,
-                             int64_t span, int64_t P, int64_t L, int32_t *cx, int32_t *cy,
+template <typename IT>
+cudaError_t launch_partition(const IT *rp, int64_t m, int64_t nnz, int64_t d0,
+                             int64_t span, int64_t P, int64_t L, int32_t *cx, IT *cy,
                              float *zero_C, int64_t ldc, int64_t row_base, int32_t K,
                              int32_t tail_row, float *tail, cudaStream_t s) {
     const int64_t n = P + 1;
     const int64_t blocks = (n + kBlock - 1) / kBlock;
-    partition_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(rp, m, nnz, d0, span, P, L, cx, cy,
+    partition_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(rp, m, nnz, d0, span, P, L, cx, cy,
                                                          zero_C, ldc, row_base, K, tail_row,
                                                          tail);
     return cudaGetLastError();
@@ -68,29 +71,31 @@ cudaError_t launch_partition(const int32_t *rp, int64_t m, int64_t nnz, int64_t 
 
 // Offline atomic fix-up: zero the rows cut by a boundary of the given schedule; one
 // warp per boundary, only the first boundary inside a row writes it.
+template <typename IT>
 __global__ void __launch_bounds__(kBlock)
-zero_split_kernel(const int32_t *__restrict__ rp, int32_t m, const int32_t *__restrict__ cx,
-                  const int32_t *__restrict__ cy, int64_t P, float *C, int64_t ldc,
+zero_split_kernel(const IT *__restrict__ rp, int32_t m, const int32_t *__restrict__ cx,
+                  const IT *__restrict__ cy, int64_t P, float *C, int64_t ldc,
                   int64_t row_base, int32_t K, int32_t tail_row, float *tail) {
     const int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (p > P) return;
     const int32_t x = cx[p];
     if (x >= m) return;
-    const int32_t start = __ldg(rp + x);
+    const IT start = __ldg(rp + x);
     if (cy[p] <= start) return;
     if (p > 0 && cx[p - 1] == x && cy[p - 1] > start) return;  // already zeroed
     float *dst = (x == tail_row) ? tail : C + ((int64_t)x - row_base) * ldc;
     for (int c = lane; c < K; c += 32) dst[c] = 0.f;
 }
 
-cudaError_t launch_zero_split(const int32_t *rp, int32_t m, const int32_t *cx,
-                              const int32_t *cy, int64_t P, float *C, int64_t ldc,
+template <typename IT>
+cudaError_t launch_zero_split(const IT *rp, int32_t m, const int32_t *cx,
+                              const IT *cy, int64_t P, float *C, int64_t ldc,
                               int64_t row_base, int32_t K, int32_t tail_row, float *tail,
                               cudaStream_t s) {
     const int64_t threads = (P + 1) * 32;
     const int64_t blocks = (threads + kBlock - 1) / kBlock;
-    zero_split_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(rp, m, cx, cy, P, C, ldc, row_base,
+    zero_split_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(rp, m, cx, cy, P, C, ldc, row_base,
                                                           K, tail_row, tail);
     return cudaGetLastError();
 }
@@ -99,9 +104,10 @@ cudaError_t launch_zero_split(const int32_t *rp, int32_t m, const int32_t *cx,
 //   start partial (line 2) and single row (line 3): 1 atomic (line 5);
 //   else start partial: 1 atomic (line 9); end partial (line 11): 1 atomic (line 13);
 //   rows [start_row, end_row): regular stores (line 15).
+template <typename IT>
 __global__ void __launch_bounds__(kBlock)
-write_stats_kernel(const int32_t *__restrict__ rp, int32_t m, const int32_t *__restrict__ cx,
-                   const int32_t *__restrict__ cy, int64_t P,
+write_stats_kernel(const IT *__restrict__ rp, int32_t m, const int32_t *__restrict__ cx,
+                   const IT *__restrict__ cy, int64_t P,
                    unsigned long long *counts) {
     __shared__ unsigned long long s_a, s_r;
     if (threadIdx.x == 0) { s_a = 0; s_r = 0; }
@@ -109,7 +115,8 @@ write_stats_kernel(const int32_t *__restrict__ rp, int32_t m, const int32_t *__r
     const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     unsigned long long na = 0, nr = 0;
     if (p < P) {
-        const int32_t xs = cx[p], ys = cy[p], xe = cx[p + 1], ye = cy[p + 1];
+        const int32_t xs = cx[p], xe = cx[p + 1];
+        const IT ys = cy[p], ye = cy[p + 1];
         const bool sp = xs < m && ys != __ldg(rp + xs);
         const bool ep = xe < m && ye != __ldg(rp + xe);
         if (sp && xs == xe) {
@@ -129,23 +136,25 @@ write_stats_kernel(const int32_t *__restrict__ rp, int32_t m, const int32_t *__r
     if (threadIdx.x == 0) { atomicAdd(counts, s_a); atomicAdd(counts + 1, s_r); }
 }
 
-cudaError_t launch_write_stats(const int32_t *rp, int32_t m, const int32_t *cx,
-                               const int32_t *cy, int64_t P, int64_t *counts, cudaStream_t s) {
+template <typename IT>
+cudaError_t launch_write_stats(const IT *rp, int32_t m, const int32_t *cx,
+                               const IT *cy, int64_t P, int64_t *counts, cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(counts, 0, 2 * sizeof(int64_t), s);
     if (e != cudaSuccess) return e;
     const int64_t blocks = (P + kBlock - 1) / kBlock;
     if (blocks > 0)
-        write_stats_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(
+        write_stats_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(
             rp, m, cx, cy, P, reinterpret_cast<unsigned long long *>(counts));
     return cudaGetLastError();
 }
 
+template <typename IT>
 __global__ void __launch_bounds__(kBlock)
-validate_kernel(const int32_t *__restrict__ rp, const int32_t *__restrict__ col, int64_t m,
+validate_kernel(const IT *__restrict__ rp, const int32_t *__restrict__ col, int64_t m,
                 int64_t n, int64_t nnz, unsigned long long *first_bad) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i <= m) {
-        const int32_t v = rp[i];
+        const IT v = rp[i];
         bool bad = (i == 0 && v != 0) || (i == m && v != nnz) || v < 0 || v > nnz ||
                    (i > 0 && rp[i - 1] > v);
         if (bad) atomicMin(first_bad, (unsigned long long)i);
@@ -156,12 +165,28 @@ validate_kernel(const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
     }
 }
 
-cudaError_t launch_validate(const int32_t *rp, const int32_t *col, int64_t m, int64_t n,
+template <typename IT>
+cudaError_t launch_validate(const IT *rp, const int32_t *col, int64_t m, int64_t n,
                             int64_t nnz, unsigned long long *first_bad, cudaStream_t s) {
     const int64_t work = (m + 1 > nnz ? m + 1 : nnz);
     const int64_t blocks = (work + kBlock - 1) / kBlock;
-    validate_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(rp, col, m, n, nnz, first_bad);
+    validate_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(rp, col, m, n, nnz, first_bad);
     return cudaGetLastError();
 }
+
+#define MPS_INST_PARTITION(IT)                                                               \
+    template cudaError_t launch_partition<IT>(const IT *, int64_t, int64_t, int64_t, int64_t,  \
+                                              int64_t, int64_t, int32_t *, IT *, float *,      \
+                                              int64_t, int64_t, int32_t, int32_t, float *,     \
+                                              cudaStream_t);                                   \
+    template cudaError_t launch_zero_split<IT>(const IT *, int32_t, const int32_t *,           \
+                                               const IT *, int64_t, float *, int64_t, int64_t, \
+                                               int32_t, int32_t, float *, cudaStream_t);       \
+    template cudaError_t launch_write_stats<IT>(const IT *, int32_t, const int32_t *,          \
+                                                const IT *, int64_t, int64_t *, cudaStream_t); \
+    template cudaError_t launch_validate<IT>(const IT *, const int32_t *, int64_t, int64_t,    \
+                                             int64_t, unsigned long long *, cudaStream_t);
+MPS_INST_PARTITION(int32_t)
+MPS_INST_PARTITION(int64_t)
 
 }  // namespace mps

@@ -56,15 +56,16 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_UL_DIV
 #define MPS_UL_DIV 1
 #endif
-template <int W, int V, typename TB>
+template <int W, int V, typename TB, typename IT>
 constexpr int seg_min_blocks() {
-    return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2
-                                                      : (sizeof(TB) == 2 ? MPS_MINB_BF16 : MPS_MINB_F32);
+    // int64 indices (NEXT-4) need more registers for the nnz coordinates: 2 CTAs/SM
+    return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8 || sizeof(IT) == 8)
+               ? 2 : (sizeof(TB) == 2 ? MPS_MINB_BF16 : MPS_MINB_F32);
 }
 
-template <int W, int V, int NR, typename TB, int FIX>
-__global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB>()))
-segment_kernel(const SegArgs a) {
+template <int W, int V, int NR, typename TB, int FIX, typename IT>
+__global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB, IT>()))
+segment_kernel(const SegArgsT<IT> a) {
     using BV = BVec<TB, W>;
     using raw_t = typename BV::raw;
     static_assert(NR == 1 || V == 1, "several rows per instruction only for one slot");
@@ -98,7 +99,7 @@ segment_kernel(const SegArgs a) {
     const int64_t wid = (int64_t)blockIdx.x * kWarps + warp;
     const int64_t wstride = (int64_t)gridDim.x * kWarps;
 
-    const int32_t *__restrict__ rp = a.rp;
+    const IT *__restrict__ rp = a.rp;
     const int32_t *__restrict__ col = a.col;
     const float *__restrict__ val = a.val;
     const char *__restrict__ Bc = reinterpret_cast<const char *>(a.B);
@@ -120,22 +121,23 @@ segment_kernel(const SegArgs a) {
 
     // chunk origin of a segment: nnz index whose col address is 16-B aligned (TMA) or
     // simply ys rounded down to a multiple of 4 (direct mode)
-    auto seg_origin = [&](int ys) -> int {
-        if (direct) return ys & ~3;
-        return ys - (int)(((uintptr_t)(col + ys) & 15u) >> 2);
+    auto seg_origin = [&](IT ys) -> IT {
+        if (direct) return ys & ~(IT)3;
+        return ys - (IT)(((uintptr_t)(col + ys) & 15u) >> 2);
     };
     // TMA may not read past the last 16-B boundary inside [.., nnz_end)
     const int64_t lim4 = a.nnz_end - (int64_t)(((uintptr_t)(col + a.nnz_end) & 15u) >> 2);
 
     // ---------------- producer: one chunk ahead, across this warp's segments ----------
     int64_t pseg = wid;
-    int pys = 0, pye = 0, psb = 0, pk = 0, pnch = 0, pbuf = 0;
+    IT pys = 0, pye = 0, psb = 0;
+    int pk = 0, pnch = 0, pbuf = 0;
     auto prod_load_seg = [&]() {
         if (pseg < a.P) {
             pys = __ldg(a.cy + pseg);
             pye = __ldg(a.cy + pseg + 1);
             psb = seg_origin(pys);
-            pnch = pye > pys ? (pye - psb + kCH - 1) / kCH : 0;
+            pnch = pye > pys ? (int)((pye - psb + kCH - 1) / kCH) : 0;
         }
         pk = 0;
     };
@@ -145,8 +147,8 @@ segment_kernel(const SegArgs a) {
             prod_load_seg();
         }
         if (pseg >= a.P) return;
-        const int cb = psb + pk * kCH;
-        const int hi = min(pye, cb + kCH);
+        const IT cb = psb + (IT)pk * kCH;
+        const IT hi = pye < cb + kCH ? pye : cb + kCH;
         int32_t *dc = st.col[pbuf];
         float *dv = st.val[pbuf];
         if (!direct) {
@@ -161,7 +163,7 @@ segment_kernel(const SegArgs a) {
                     tma_load_1d(dv, val + cb, bytes, &bars[warp][pbuf], pol_first);
                 }
             }
-            const int rem = hi - (int)ce;   // < 4 entries at the very end of the array
+            const int rem = (int)(hi - (IT)ce);   // < 4 entries at the very end of the array
             if (lane < rem) {
                 dc[ce - cb + lane] = col[ce + lane];
                 dv[ce - cb + lane] = val[ce + lane];
@@ -184,17 +186,20 @@ segment_kernel(const SegArgs a) {
     int cbuf = 0;
 
     for (int64_t seg = wid; seg < a.P; seg += wstride) {
-        const int xs = __ldg(a.cx + seg), ys = __ldg(a.cy + seg);
-        const int xe = __ldg(a.cx + seg + 1), ye = __ldg(a.cy + seg + 1);
-        const int sb = seg_origin(ys);
-        const int nch = ye > ys ? (ye - sb + kCH - 1) / kCH : 0;
+        const int xs = __ldg(a.cx + seg);
+        const IT ys = __ldg(a.cy + seg);
+        const int xe = __ldg(a.cx + seg + 1);
+        const IT ye = __ldg(a.cy + seg + 1);
+        const IT sb = seg_origin(ys);
+        const int nch = ye > ys ? (int)((ye - sb + kCH - 1) / kCH) : 0;
 
         // row_ptr window: lane l holds rp[wb + l]
         int wb = xs;
-        int win = (wb + lane <= m) ? __ldg(rp + wb + lane) : 0x7fffffff;
-        const int rp_xs = __shfl_sync(0xffffffffu, win, 0);
-        int rend = __shfl_sync(0xffffffffu, win, 1);   // rp[r + 1]
-        int rbeg = rp_xs;                               // rp[r]
+        constexpr IT kInf = sizeof(IT) == 8 ? (IT)0x7fffffffffffffffll : (IT)0x7fffffff;
+        IT win = (wb + lane <= m) ? __ldg(rp + wb + lane) : kInf;
+        const IT rp_xs = __shfl_sync(0xffffffffu, win, 0);
+        IT rend = __shfl_sync(0xffffffffu, win, 1);   // rp[r + 1]
+        IT rbeg = rp_xs;                               // rp[r]
         const bool start_in = xs < m && ys > rp_xs;     // Alg. 2 line 2 (start_nz != 0)
         int r = xs;
 
@@ -260,7 +265,7 @@ segment_kernel(const SegArgs a) {
             int idx = r + 1 - wb;
             if (idx >= 32) {
                 wb = r;
-                win = (wb + lane <= m) ? __ldg(rp + wb + lane) : 0x7fffffff;
+                win = (wb + lane <= m) ? __ldg(rp + wb + lane) : kInf;
                 idx = 1;
             }
             rbeg = rend;
@@ -289,14 +294,14 @@ segment_kernel(const SegArgs a) {
             __syncwarp();
             produce();                  // next chunk into the other buffer
             if (direct) __syncwarp();
-            const int cb = sb + k * kCH;
+            const IT cb = sb + (IT)k * kCH;
             const int32_t *sc = st.col[cbuf];
             const float *sv = st.val[cbuf];
-            int q = ys - cb;
-            q = q > 0 ? (q / U) * U : 0;
-            const int qend = min(kCH, ye - cb);
+            int q = ys > cb ? (int)(ys - cb) : 0;
+            q = (q / U) * U;
+            const int qend = ye - cb < (IT)kCH ? (int)(ye - cb) : kCH;
             for (; q < qend; q += U) {
-                const int j0 = cb + q;
+                const IT j0 = cb + q;
                 raw_t bv[UL][V];
                 const bool full = j0 >= ys && j0 + U <= ye;
                 // my non-zeros of this batch: u = i*NR + grp (i < UL).  Column indices
@@ -320,7 +325,7 @@ segment_kernel(const SegArgs a) {
                 if (!full) {
 #pragma unroll
                     for (int i = 0; i < UL; ++i) {
-                        const int j = j0 + i * NR + grp;
+                        const IT j = j0 + i * NR + grp;
                         cid[i] = (j >= ys && j < ye) ? cid[i] : 0u;
                     }
                 }
@@ -368,14 +373,14 @@ segment_kernel(const SegArgs a) {
                     float vl[UL];
 #pragma unroll
                     for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
-                    int jc = j0 > ys ? j0 : ys;                  // next non-zero to consume
-                    const int jend = (j0 + U < ye) ? j0 + U : ye;
+                    IT jc = j0 > ys ? j0 : ys;                   // next non-zero to consume
+                    const IT jend = (j0 + U < ye) ? j0 + U : ye;
                     while (jc < jend) {
                         while (jc >= rend) finish_row();          // rows ending before jc
-                        const int lim = rend < jend ? rend : jend;  // row r's part: [jc, lim)
+                        const IT lim = rend < jend ? rend : jend;   // row r's part: [jc, lim)
 #pragma unroll
                         for (int i = 0; i < UL; ++i) {
-                            const int j = j0 + i * NR + grp;
+                            const IT j = j0 + i * NR + grp;
                             if (j >= jc && j < lim) fma_row(vl[i], bv[i]);
                         }
                         jc = lim;
@@ -400,8 +405,8 @@ segment_kernel(const SegArgs a) {
     }
 }
 
-template <int W, int V, int NR, typename TB, int FIX>
-static cudaError_t launch_seg(const SegArgs &a, cudaStream_t s) {
+template <int W, int V, int NR, typename TB, int FIX, typename IT>
+static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     static int blocks_per_sm = 0;
     if (blocks_per_sm == 0) {
         // the staging buffers need the large shared-memory carveout for
@@ -413,12 +418,12 @@ static cudaError_t launch_seg(const SegArgs &a, cudaStream_t s) {
         }();
         cudaError_t e = cudaSuccess;
         if (carve >= 0) {
-            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX>,
+            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT>,
                                      cudaFuncAttributePreferredSharedMemoryCarveout, carve);
             if (e != cudaSuccess) return e;
         }
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX>, kBlock, 0);
+            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX, IT>, kBlock, 0);
         if (e != cudaSuccess) return e;
         if (blocks_per_sm < 1) blocks_per_sm = 1;
     }
@@ -427,41 +432,41 @@ static cudaError_t launch_seg(const SegArgs &a, cudaStream_t s) {
     const int64_t cap = (int64_t)blocks_per_sm * num_sms();
     const int64_t grid = need < cap ? need : cap;
     if (grid <= 0) return cudaSuccess;
-    segment_kernel<W, V, NR, TB, FIX><<<(unsigned)grid, kBlock, 0, s>>>(a);
+    segment_kernel<W, V, NR, TB, FIX, IT><<<(unsigned)grid, kBlock, 0, s>>>(a);
     return cudaGetLastError();
 }
 
 // (W, V, NR) dispatch.  NR > 1 only with V == 1.
-template <typename TB, int FIX, int W>
-static cudaError_t dispatch_v(const SegArgs &a, int V, int NR, cudaStream_t s) {
+template <typename TB, int FIX, int W, typename IT>
+static cudaError_t dispatch_v(const SegArgsT<IT> &a, int V, int NR, cudaStream_t s) {
     if (V == 1) {
         switch (NR) {
-        case 1: return launch_seg<W, 1, 1, TB, FIX>(a, s);
-        case 2: return launch_seg<W, 1, 2, TB, FIX>(a, s);
-        case 4: return launch_seg<W, 1, 4, TB, FIX>(a, s);
-        case 8: return launch_seg<W, 1, 8, TB, FIX>(a, s);
-        case 16: return launch_seg<W, 1, 16, TB, FIX>(a, s);
-        case 32: return launch_seg<W, 1, 32, TB, FIX>(a, s);
+        case 1: return launch_seg<W, 1, 1, TB, FIX, IT>(a, s);
+        case 2: return launch_seg<W, 1, 2, TB, FIX, IT>(a, s);
+        case 4: return launch_seg<W, 1, 4, TB, FIX, IT>(a, s);
+        case 8: return launch_seg<W, 1, 8, TB, FIX, IT>(a, s);
+        case 16: return launch_seg<W, 1, 16, TB, FIX, IT>(a, s);
+        case 32: return launch_seg<W, 1, 32, TB, FIX, IT>(a, s);
         default: return cudaErrorInvalidValue;
         }
     }
     if (NR != 1) return cudaErrorInvalidValue;
     switch (V) {
-    case 2: return launch_seg<W, 2, 1, TB, FIX>(a, s);
-    case 3: return launch_seg<W, 3, 1, TB, FIX>(a, s);
-    case 4: return launch_seg<W, 4, 1, TB, FIX>(a, s);
+    case 2: return launch_seg<W, 2, 1, TB, FIX, IT>(a, s);
+    case 3: return launch_seg<W, 3, 1, TB, FIX, IT>(a, s);
+    case 4: return launch_seg<W, 4, 1, TB, FIX, IT>(a, s);
     default: return cudaErrorInvalidValue;
     }
 }
 
-template <typename TB, int FIX>
-static cudaError_t dispatch_w(const SegArgs &a, int W, int V, int NR, cudaStream_t s) {
+template <typename TB, int FIX, typename IT>
+static cudaError_t dispatch_w(const SegArgsT<IT> &a, int W, int V, int NR, cudaStream_t s) {
     switch (W) {
-    case 1: return dispatch_v<TB, FIX, 1>(a, V, NR, s);
-    case 2: return dispatch_v<TB, FIX, 2>(a, V, NR, s);
-    case 4: return dispatch_v<TB, FIX, 4>(a, V, NR, s);
+    case 1: return dispatch_v<TB, FIX, 1, IT>(a, V, NR, s);
+    case 2: return dispatch_v<TB, FIX, 2, IT>(a, V, NR, s);
+    case 4: return dispatch_v<TB, FIX, 4, IT>(a, V, NR, s);
     case 8:
-        if constexpr (sizeof(TB) == 2) return dispatch_v<TB, FIX, 8>(a, V, NR, s);
+        if constexpr (sizeof(TB) == 2) return dispatch_v<TB, FIX, 8, IT>(a, V, NR, s);
         return cudaErrorInvalidValue;
     default: return cudaErrorInvalidValue;
     }

@@ -4,12 +4,18 @@
 
 namespace mps {
 
+// one translation unit per (index type, B dtype, fix-up) so the build parallelises
 cudaError_t launch_segments_f32_atomic(const SegArgs &a, int W, int V, int NR, cudaStream_t s);
 cudaError_t launch_segments_f32_carry(const SegArgs &a, int W, int V, int NR, cudaStream_t s);
 cudaError_t launch_segments_bf16_atomic(const SegArgs &a, int W, int V, int NR, cudaStream_t s);
 cudaError_t launch_segments_bf16_carry(const SegArgs &a, int W, int V, int NR, cudaStream_t s);
+cudaError_t launch_segments_f32_atomic(const SegArgs64 &a, int W, int V, int NR, cudaStream_t s);
+cudaError_t launch_segments_f32_carry(const SegArgs64 &a, int W, int V, int NR, cudaStream_t s);
+cudaError_t launch_segments_bf16_atomic(const SegArgs64 &a, int W, int V, int NR, cudaStream_t s);
+cudaError_t launch_segments_bf16_carry(const SegArgs64 &a, int W, int V, int NR, cudaStream_t s);
 
-cudaError_t launch_segments(const SegArgs &a, int b_dtype, int W, int V, int NR, int fix,
+template <typename IT>
+cudaError_t launch_segments(const SegArgsT<IT> &a, int b_dtype, int W, int V, int NR, int fix,
                             cudaStream_t s) {
     if (b_dtype == MPS_DT_F32)
         return fix == FIX_CARRY ? launch_segments_f32_carry(a, W, V, NR, s)
@@ -22,14 +28,15 @@ cudaError_t launch_segments(const SegArgs &a, int b_dtype, int W, int V, int NR,
 // inside a row r, the row's pieces are the end piece of segment p-1 (slot 1) and the
 // start pieces (slot 0) of segments p, p+1, ... that start inside r.  They are summed
 // in segment order (deterministic) and stored -- no zero-initialisation needed.
+template <typename IT>
 __global__ void __launch_bounds__(kBlock)
-carry_reduce_kernel(const SegArgs a) {
+carry_reduce_kernel(const SegArgsT<IT> a) {
     const int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (p > a.P) return;
     const int32_t r = a.cx[p];
     if (r >= a.m) return;
-    const int32_t rs = __ldg(a.rp + r);
+    const IT rs = __ldg(a.rp + r);
     if (a.cy[p] <= rs) return;                                 // not inside row r
     if (p > 0 && a.cx[p - 1] == r && a.cy[p - 1] > rs) return; // not the first boundary
     // chain length: segments s = p .. q-1 start inside row r (s < P)
@@ -78,34 +85,37 @@ carry_reduce_kernel(const SegArgs a) {
     }
 }
 
-cudaError_t launch_carry_reduce(const SegArgs &a, cudaStream_t s) {
+template <typename IT>
+cudaError_t launch_carry_reduce(const SegArgsT<IT> &a, cudaStream_t s) {
     const int64_t threads = (a.P + 1) * 32;
     const int64_t blocks = (threads + kBlock - 1) / kBlock;
-    carry_reduce_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(a);
+    carry_reduce_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(a);
     return cudaGetLastError();
 }
 
 // Epilogue for the rows cut by a schedule boundary in atomic mode: they are final only
 // after every partial sum has landed, so the ReLU runs here, once per cut row (one warp
 // per first boundary inside the row).
+template <typename IT>
 __global__ void __launch_bounds__(kBlock)
-relu_split_kernel(const SegArgs a) {
+relu_split_kernel(const SegArgsT<IT> a) {
     const int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (p > a.P) return;
     const int32_t r = a.cx[p];
     if (r >= a.m || r == a.tail_row) return;
-    const int32_t rs = __ldg(a.rp + r);
+    const IT rs = __ldg(a.rp + r);
     if (a.cy[p] <= rs) return;
     if (p > 0 && a.cx[p - 1] == r && a.cy[p - 1] > rs) return;
     float *dst = a.C + ((int64_t)r - a.row_base) * a.ldc;
     for (int c = lane; c < a.K; c += 32) dst[c] = fmaxf(dst[c], 0.f);
 }
 
-cudaError_t launch_relu_split(const SegArgs &a, cudaStream_t s) {
+template <typename IT>
+cudaError_t launch_relu_split(const SegArgsT<IT> &a, cudaStream_t s) {
     const int64_t threads = (a.P + 1) * 32;
     const int64_t blocks = (threads + kBlock - 1) / kBlock;
-    relu_split_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(a);
+    relu_split_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -132,5 +142,13 @@ cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx
     apply_tails_kernel<<<1, kBlock, 0, s>>>(tails, K, t, n, row);
     return cudaGetLastError();
 }
+
+#define MPS_INST_SPMM(IT)                                                                     \
+    template cudaError_t launch_segments<IT>(const SegArgsT<IT> &, int, int, int, int, int,     \
+                                             cudaStream_t);                                     \
+    template cudaError_t launch_carry_reduce<IT>(const SegArgsT<IT> &, cudaStream_t);          \
+    template cudaError_t launch_relu_split<IT>(const SegArgsT<IT> &, cudaStream_t);
+MPS_INST_SPMM(int32_t)
+MPS_INST_SPMM(int64_t)
 
 }  // namespace mps

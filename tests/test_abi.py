@@ -77,3 +77,24 @@ def test_shard_bounds_match_oracle(world):
     g = G.random_csr(9, 9, rl, 1)
     X, Y, T = M.shard_bounds(g.row_ptr, world)
     assert np.array_equal(T, O.shard(g.row_ptr, world)[2])
+
+
+def test_plan64_host_only():
+    """NEXT-4: mps_plan64 lifts the 2^31 limit on M = m + nnz (same Alg. 1 sizing as
+    the oracle); m >= 2^31 stays unsupported (rows are int32)."""
+    for (m, nnz, cost, pmin) in [(10, 2 ** 31, 2048, 1), (2 ** 31 - 1, 2 ** 40, 4096, 1184),
+                                 (5, 0, 7, 1), (232965, 114615892, 2048, 1184)]:
+        assert M.plan(m, nnz, 64, 0, cost, pmin, wide=True) == O.plan(m, nnz, cost, pmin)
+    P, L = ctypes.c_int64(), ctypes.c_int64()
+    with pytest.raises(M.MpsError) as e:
+        M.mps_plan64(2 ** 31, 0, 8, 0, 0, 0, ctypes.byref(P), ctypes.byref(L))
+    assert e.value.status == M.MPS_ERR_UNSUPPORTED
+    a = M.mps_csr64(2 ** 31, 4, 0, None, None, None)
+    nb = ctypes.c_size_t()
+    with pytest.raises(M.MpsError) as e:
+        M.mps_spmm64_online_workspace_bytes(ctypes.byref(a), 16, 0, 0, 0, 1, ctypes.byref(nb))
+    assert e.value.status == M.MPS_ERR_UNSUPPORTED
+    a = M.mps_csr64(1000, 1000, 3 * 2 ** 30, None, None, None)
+    M.mps_spmm64_online_workspace_bytes(ctypes.byref(a), 16, 0, 0, 0, 1, ctypes.byref(nb))
+    Pp, Lp = M.plan(1000, 3 * 2 ** 30, 16, 0, 0, 0, wide=True)
+    assert nb.value >= (Pp + 1) * 12       # int32 coord_x + int64 coord_y

@@ -49,3 +49,22 @@ def test_random_csr_adversarial():
     g = G.random_csr(6, 4, rl, seed=3, canonical=False)
     assert np.array_equal(np.diff(g.row_ptr), rl)
     assert set(np.unique(g.val).tolist()) <= {1.0, 2.0, 3.0}
+
+
+def test_wide_generator_host_equals_device_formula():
+    """NEXT-4 wide graphs: the numpy (host) and torch (device) evaluations of the
+    counter-based hash give the same bytes; splitmix64's first output from state 0 is
+    the published 0xE220A8397B1DCDAF."""
+    import torch
+    assert int(G._mix_np(np.uint64(0))) == 0xE220A8397B1DCDAF
+    j = np.arange(0, 100000, dtype=np.int64) * 104729 + (1 << 31) - 5
+    c, v = G.wide_cols_vals_host(j, 999983, 11)
+    ct, vt = G.wide_cols_vals_device(0, 999983, 11, device="cpu")  # empty, exercises the API
+    assert ct.numel() == 0
+    jt = torch.from_numpy(j)
+    assert np.array_equal(c, (G._h31_torch(12, jt) % 999983).to(torch.int32).numpy())
+    assert np.array_equal(v, (1 + G._h31_torch(13, jt) % 3).to(torch.float32).numpy())
+    assert c.min() >= 0 and c.max() < 999983 and set(np.unique(v)) == {1.0, 2.0, 3.0}
+    rp = G.wide_row_ptr(1000, 2048, 3, evil=[(7, 10 ** 6)])
+    assert rp.dtype == np.int64 and rp[0] == 0 and np.all(np.diff(rp) >= 0)
+    assert rp[8] - rp[7] == 10 ** 6 and np.diff(rp).max() == 10 ** 6

@@ -246,6 +246,52 @@ def test_o4_sub_range_diagonals():
     assert np.array_equal(cx, xs[dd]) and np.array_equal(cy, ys[dd])
 
 
+def test_o4_partition64_small_equals_int32_partition():
+    """NEXT-4: the int64-offset partition is the same Alg. 1 closed form."""
+    rs = np.random.RandomState(17)
+    for trial in range(60):
+        g = rand_graph(rs, rs.randint(0, 150), 40, 10, seed=trial)
+        M = g.m + g.nnz
+        P = int(rs.randint(1, 30))
+        L = -(-M // P)
+        cx, cy = O.partition(g.row_ptr, P, L)
+        cx64, cy64 = O.partition64(g.row_ptr.astype(np.int64), P, L)
+        assert cy64.dtype == np.int64
+        assert np.array_equal(cx, cx64) and np.array_equal(cy.astype(np.int64), cy64)
+
+
+def test_o4_partition64_beyond_2p31_matches_searchsorted():
+    """NEXT-4: m + nnz > 2^31.  x_p = max{x : x + RP[x] <= d_p} (reading R4) computed by
+    numpy's searchsorted over the strictly increasing s(x) = x + RP[x] -- a library
+    primitive, not the oracle's bisection -- and the unique-point property
+    RP[x] <= y <= RP[x+1] (reading R5), including diagonals at the 2^31 boundary."""
+    rs = np.random.RandomState(18)
+    m = 200_000
+    rl = rs.randint(0, 40_000, size=m).astype(np.int64)
+    rl[rs.randint(m, size=5)] = 3_000_000_000 // 5   # a few rows past 2^31 on their own
+    rl[rl % 7 == 0] = 0
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(rl, out=rp[1:])
+    nnz = int(rp[-1])
+    assert m + nnz > 2 ** 32
+    s = np.arange(m + 1, dtype=np.int64) + rp
+    P = 5000
+    L = -(-(m + nnz) // P)
+    cx, cy = O.partition64(rp, P, L)
+    d = np.minimum(np.arange(P + 1, dtype=np.int64) * L, m + nnz)
+    x_ref = np.searchsorted(s, d, side="right") - 1
+    assert np.array_equal(cx.astype(np.int64), x_ref)
+    assert np.array_equal(cy, d - x_ref)
+    assert np.all(rp[cx] <= cy)
+    inner = cx < m
+    assert np.all(cy[inner] <= rp[cx[inner] + 1])
+    # single diagonals straddling 2^31 (through the sub-range form of line 4)
+    for dd in (2 ** 31 - 1, 2 ** 31, 2 ** 31 + 1, 2 ** 32 + 12345):
+        bx, by = O.partition64(rp, 1, 0, dd, dd)
+        xr = int(np.searchsorted(s, dd, side="right") - 1)
+        assert (int(bx[0]), int(by[0])) == (xr, dd - xr)
+
+
 # --------------------------------------------------------------------------------
 # O6: Alg. 2 (P:100-131)
 # --------------------------------------------------------------------------------
