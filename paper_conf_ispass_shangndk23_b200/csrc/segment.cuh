@@ -56,11 +56,15 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_UL_DIV
 #define MPS_UL_DIV 1
 #endif
+#ifndef MPS_MINB_I64
+#define MPS_MINB_I64 3
+#endif
 template <int W, int V, typename TB, typename IT>
 constexpr int seg_min_blocks() {
-    // int64 indices (NEXT-4) need more registers for the nnz coordinates: 2 CTAs/SM
-    return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8 || sizeof(IT) == 8)
-               ? 2 : (sizeof(TB) == 2 ? MPS_MINB_BF16 : MPS_MINB_F32);
+    // int64 indices (NEXT-4): fp32 B measured best at 3 CTAs/SM with a few spills
+    // (profiles/r01/next4), bf16 B keeps the int32 choice
+    return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2
+           : (sizeof(TB) == 2 ? MPS_MINB_BF16 : (sizeof(IT) == 8 ? MPS_MINB_I64 : MPS_MINB_F32));
 }
 
 template <int W, int V, int NR, typename TB, int FIX, typename IT>
@@ -130,14 +134,16 @@ segment_kernel(const SegArgsT<IT> a) {
 
     // ---------------- producer: one chunk ahead, across this warp's segments ----------
     int64_t pseg = wid;
-    IT pys = 0, pye = 0, psb = 0;
+    IT psb = 0;                          // chunk origin of the producer's segment
+    int pys = 0, pye = 0;                // its non-zero range, relative to psb
     int pk = 0, pnch = 0, pbuf = 0;
     auto prod_load_seg = [&]() {
         if (pseg < a.P) {
-            pys = __ldg(a.cy + pseg);
-            pye = __ldg(a.cy + pseg + 1);
-            psb = seg_origin(pys);
-            pnch = pye > pys ? (int)((pye - psb + kCH - 1) / kCH) : 0;
+            const IT ys_ = __ldg(a.cy + pseg), ye_ = __ldg(a.cy + pseg + 1);
+            psb = seg_origin(ys_);
+            pys = (int)(ys_ - psb);
+            pye = (int)(ye_ - psb);
+            pnch = pye > pys ? (pye + kCH - 1) / kCH : 0;
         }
         pk = 0;
     };
@@ -147,8 +153,10 @@ segment_kernel(const SegArgsT<IT> a) {
             prod_load_seg();
         }
         if (pseg >= a.P) return;
-        const IT cb = psb + (IT)pk * kCH;
-        const IT hi = pye < cb + kCH ? pye : cb + kCH;
+        const int cbr = pk * kCH;
+        const int hir = min(pye, cbr + kCH);
+        const IT cb = psb + cbr;
+        const IT hi = psb + hir;
         int32_t *dc = st.col[pbuf];
         float *dv = st.val[pbuf];
         if (!direct) {
@@ -169,8 +177,8 @@ segment_kernel(const SegArgsT<IT> a) {
                 dv[ce - cb + lane] = val[ce + lane];
             }
         } else {
-            for (int t = lane; cb + t < hi; t += 32) {
-                if (cb + t >= pys) {
+            for (int t = lane; cbr + t < hir; t += 32) {
+                if (cbr + t >= pys) {
                     dc[t] = __ldg(col + cb + t);
                     dv[t] = __ldg(val + cb + t);
                 }
@@ -187,19 +195,36 @@ segment_kernel(const SegArgsT<IT> a) {
 
     for (int64_t seg = wid; seg < a.P; seg += wstride) {
         const int xs = __ldg(a.cx + seg);
-        const IT ys = __ldg(a.cy + seg);
+        const IT ys64 = __ldg(a.cy + seg);
         const int xe = __ldg(a.cx + seg + 1);
-        const IT ye = __ldg(a.cy + seg + 1);
-        const IT sb = seg_origin(ys);
-        const int nch = ye > ys ? (int)((ye - sb + kCH - 1) / kCH) : 0;
+        const IT ye64 = __ldg(a.cy + seg + 1);
+        const IT sb64 = seg_origin(ys64);
+        const int nch = ye64 > ys64 ? (int)((ye64 - sb64 + kCH - 1) / kCH) : 0;
+
+        // Non-zero positions inside the segment are handled as 32-bit offsets from
+        // `base` (0 for int32 indices; the segment's chunk origin for int64 indices,
+        // NEXT-4).  Row offsets outside the segment are clamped to [-1, ye + 1], which
+        // keeps every comparison the walk makes (all against positions in [ys, ye]).
+        const IT base = sizeof(IT) == 8 ? sb64 : (IT)0;
+        const IT hic = ye64 - base + 1;
+        auto rel = [&](IT v) -> int {
+            if constexpr (sizeof(IT) == 8) {
+                IT d = v - base;
+                d = d < (IT)-1 ? (IT)-1 : (d > hic ? hic : d);
+                return (int)d;
+            } else {
+                return (int)v;
+            }
+        };
+        const int ys = rel(ys64), ye = rel(ye64), sb = rel(sb64);
 
         // row_ptr window: lane l holds rp[wb + l]
         int wb = xs;
         constexpr IT kInf = sizeof(IT) == 8 ? (IT)0x7fffffffffffffffll : (IT)0x7fffffff;
-        IT win = (wb + lane <= m) ? __ldg(rp + wb + lane) : kInf;
-        const IT rp_xs = __shfl_sync(0xffffffffu, win, 0);
-        IT rend = __shfl_sync(0xffffffffu, win, 1);   // rp[r + 1]
-        IT rbeg = rp_xs;                               // rp[r]
+        int win = rel((wb + lane <= m) ? __ldg(rp + wb + lane) : kInf);
+        const int rp_xs = __shfl_sync(0xffffffffu, win, 0);
+        int rend = __shfl_sync(0xffffffffu, win, 1);   // rp[r + 1]
+        int rbeg = rp_xs;                               // rp[r]
         const bool start_in = xs < m && ys > rp_xs;     // Alg. 2 line 2 (start_nz != 0)
         int r = xs;
 
@@ -265,7 +290,7 @@ segment_kernel(const SegArgsT<IT> a) {
             int idx = r + 1 - wb;
             if (idx >= 32) {
                 wb = r;
-                win = (wb + lane <= m) ? __ldg(rp + wb + lane) : kInf;
+                win = rel((wb + lane <= m) ? __ldg(rp + wb + lane) : kInf);
                 idx = 1;
             }
             rbeg = rend;
@@ -294,14 +319,14 @@ segment_kernel(const SegArgsT<IT> a) {
             __syncwarp();
             produce();                  // next chunk into the other buffer
             if (direct) __syncwarp();
-            const IT cb = sb + (IT)k * kCH;
+            const int cb = sb + k * kCH;
             const int32_t *sc = st.col[cbuf];
             const float *sv = st.val[cbuf];
-            int q = ys > cb ? (int)(ys - cb) : 0;
-            q = (q / U) * U;
-            const int qend = ye - cb < (IT)kCH ? (int)(ye - cb) : kCH;
+            int q = ys - cb;
+            q = q > 0 ? (q / U) * U : 0;
+            const int qend = min(kCH, ye - cb);
             for (; q < qend; q += U) {
-                const IT j0 = cb + q;
+                const int j0 = cb + q;
                 raw_t bv[UL][V];
                 const bool full = j0 >= ys && j0 + U <= ye;
                 // my non-zeros of this batch: u = i*NR + grp (i < UL).  Column indices
@@ -325,7 +350,7 @@ segment_kernel(const SegArgsT<IT> a) {
                 if (!full) {
 #pragma unroll
                     for (int i = 0; i < UL; ++i) {
-                        const IT j = j0 + i * NR + grp;
+                        const int j = j0 + i * NR + grp;
                         cid[i] = (j >= ys && j < ye) ? cid[i] : 0u;
                     }
                 }
@@ -373,14 +398,14 @@ segment_kernel(const SegArgsT<IT> a) {
                     float vl[UL];
 #pragma unroll
                     for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
-                    IT jc = j0 > ys ? j0 : ys;                   // next non-zero to consume
-                    const IT jend = (j0 + U < ye) ? j0 + U : ye;
+                    int jc = j0 > ys ? j0 : ys;                  // next non-zero to consume
+                    const int jend = (j0 + U < ye) ? j0 + U : ye;
                     while (jc < jend) {
                         while (jc >= rend) finish_row();          // rows ending before jc
-                        const IT lim = rend < jend ? rend : jend;   // row r's part: [jc, lim)
+                        const int lim = rend < jend ? rend : jend;  // row r's part: [jc, lim)
 #pragma unroll
                         for (int i = 0; i < UL; ++i) {
-                            const IT j = j0 + i * NR + grp;
+                            const int j = j0 + i * NR + grp;
                             if (j >= jc && j < lim) fma_row(vl[i], bv[i]);
                         }
                         jc = lim;
