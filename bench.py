@@ -185,6 +185,65 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+# input feature width F of the combination X*W per workload (the datasets' feature sizes;
+# synthetic R-MAT: 64)
+FEATURES = {"cora": 1433, "pubmed": 500, "reddit": 602, "products": 100, "rmat": 64}
+
+
+def xw_replication(M, g, K, rank, world, dev, stream):
+    """NEXT-3 multi-GPU: produce the replicated B (bf16) from row-sharded X.
+    fused: ONE kernel per rank (mps_xw_bf16_bcast) computes its row block of X*W and stores
+    it into every rank's replica over NVLink (CUDA IPC peer pointers);
+    unfused: the same GEMM into the local block, then NCCL all_gather_into_tensor.
+    Times are CUDA events on the launching stream, max over ranks, best of 3."""
+    import torch
+    import torch.distributed as dist
+    F = FEATURES.get(g.name.split("-")[0], 64)
+    ldx = -(-F // 8) * 8
+    r0, r1 = M.row_block(g.n, world, rank)
+    gen = torch.Generator(device="cpu").manual_seed(1000 + rank)
+    X = torch.zeros((max(r1 - r0, 1), ldx), dtype=torch.bfloat16)
+    X[:, :F] = torch.randn(X.shape[0], F, generator=gen).to(torch.bfloat16)
+    X = X.to(dev)[: r1 - r0, :F]
+    Wt = torch.zeros((K, ldx), dtype=torch.bfloat16)
+    Wt[:, :F] = (torch.randn(K, F, generator=torch.Generator().manual_seed(7)) / F ** 0.5)
+    Wt = Wt.to(dev)[:, :F]
+    rep = M.PeerReplicas(g.n, K, rank, world, dev)
+    nccl = dist.get_backend() == "nccl"
+    per = -(-g.n // world)
+    full = torch.empty((per * world, K), dtype=torch.bfloat16, device=dev)
+    fused, unfused = [], []
+    for _ in range(3):
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        M.xw_replicate(X, Wt, rep, sync=False)
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        dist.barrier()
+        fused.append(e0.elapsed_time(e1))
+        dist.barrier()
+        e0.record(stream)
+        M.xw_bf16(X, Wt, out=full[rank * per: rank * per + (r1 - r0)])
+        if nccl:
+            dist.all_gather_into_tensor(full, full[rank * per:(rank + 1) * per])
+        else:           # gloo (several ranks sharing one GPU in tests): host staging
+            host = torch.empty(full.shape, dtype=full.dtype)
+            dist.all_gather_into_tensor(host, full[rank * per:(rank + 1) * per].cpu())
+            full.copy_(host)
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        unfused.append(e0.elapsed_time(e1))
+    ok = torch.equal(rep.B, full[: g.n])
+    t = torch.tensor([min(fused), min(unfused), 0.0 if ok else 1.0], dtype=torch.float64,
+                     device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    rep.close()
+    return {"F": F, "fused_xw_bcast_ms": float(t[0]),
+            ("xw_then_nccl_allgather_ms" if nccl else "xw_then_gloo_allgather_ms"): float(t[1]),
+            "replicas_equal": bool(t[2] == 0.0)}
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -304,6 +363,13 @@ def main():
         dist.all_reduce(b_rep, op=dist.ReduceOp.MAX)
         b_rep_ms = float(b_rep[0])
         del Brep
+        xw_rep = None
+        if K % 16 == 0 and 16 <= K <= 256:
+            try:     # reported beside the step, never allowed to break the bench line
+                xw_rep = xw_replication(M, g, K, rank, world, dev, stream)
+            except Exception as e:  # pragma: no cover
+                xw_rep = {"error": str(e)[:200]}
+            dist.barrier()
         sh = M.ShardedSpMM(g.row_ptr, g.col_idx, g.val, g.n, K, rank, world, dev,
                            b_dtype=tdtype, fixup=args.fixup, items_per_part=args.items_per_part,
                            min_parts=args.min_parts)
@@ -484,7 +550,7 @@ def main():
                          "peak_source": peak_src},
             "b_replication": ({"ms": b_rep_ms, "bytes_per_rank_received": int(
                 (world - 1) * (-(-g.n // world)) * K * b_elt), "collective": "all_gather_into_tensor",
-                "in_step": False} if world > 1 else None),
+                "in_step": False, "fused_xw": xw_rep} if world > 1 else None),
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(launches_per_step * args.steps),

@@ -199,6 +199,31 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
 mps_status mps_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
                        int32_t N, int64_t ldw, void *B, int64_t ldb, void *stream);
 
+/* NEXT-3, multi-GPU: the combination fused with the replication of B over NVLink.  This
+ * rank's row block X (n_rows x F) times W is written as bf16 rows row_offset ..
+ * row_offset + n_rows - 1 of EVERY B replica in B_dsts_host (a HOST array of ndst
+ * device pointers, each to a full [n][ldb] bf16 replica; entry 0 should be this rank's
+ * own replica, the others peer replicas mapped with mps_ipc_open_handle).  One kernel:
+ * the epilogue of each tile stores it to all destinations, so the all-gather of B
+ * overlaps the GEMM.  Same shape rules as mps_xw_bf16, 1 <= ndst <= 16.  Completion on
+ * a peer is only guaranteed after this stream is synchronised and the ranks have met
+ * at a barrier (the caller's process group).                                        */
+mps_status mps_xw_bf16_bcast(const void *X, int64_t n_rows, int64_t F, int64_t ldx,
+                             const void *Wt, int32_t N, int64_t ldw, void *const *B_dsts_host,
+                             int32_t ndst, int64_t row_offset, int64_t ldb, void *stream);
+
+/* CUDA IPC between the ranks of one node (peer access over NVLink is enabled lazily).
+ * mps_ipc_get_handle: handle_out (mps_ipc_handle_bytes() bytes, caller-owned) names the
+ * device allocation that contains dev_ptr; *offset_out = dev_ptr - its base.  The peer
+ * opens it with mps_ipc_open_handle (base address in this process; add the offset) and
+ * unmaps it with mps_ipc_close_handle.  Errors: MPS_ERR_INVALID for NULL or non-device
+ * pointers, MPS_ERR_CUDA if the runtime refuses (e.g. a handle opened in its own
+ * process).                                                                         */
+size_t mps_ipc_handle_bytes(void);
+mps_status mps_ipc_get_handle(const void *dev_ptr, void *handle_out, int64_t *offset_out);
+mps_status mps_ipc_open_handle(const void *handle, void **base_out);
+mps_status mps_ipc_close_handle(void *base);
+
 /* Fig. 5 statistic: with the Alg. 2 write rules (lines 5, 9, 13 atomic,
  * line 15 regular) for the given schedule, counts_out[0] = #atomic row updates,
  * counts_out[1] = #regular row stores.  counts_out: device int64[2], overwritten. */

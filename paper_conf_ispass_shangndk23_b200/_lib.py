@@ -71,6 +71,11 @@ _SIGS = {
                        _p, _i32, _p, _sz, _p],
     "mps_apply_tails": [_p, _p, _p, _i32, _i32, _i32, _p, _i64, _p],
     "mps_validate_csr": [_p, _p, _p],
+    "mps_xw_bf16_bcast": [_p, _i64, _i64, _i64, _p, _i32, _i64, _p, _i32, _i64, _i64, _p],
+    "mps_ipc_handle_bytes": [],
+    "mps_ipc_get_handle": [_p, _p, _p],
+    "mps_ipc_open_handle": [_p, _p],
+    "mps_ipc_close_handle": [_p],
     "mps_plan64": [_i64, _i64, _i32, _i32, _i64, _i64, _p, _p],
     "mps_partition64": [_p, _i64, _i64, _i64, _i64, _i64, _i64, _p, _p, _p],
     "mps_spmm64_workspace_bytes": [_p, _i32, _i32, _i64, _i32, _p],
@@ -82,7 +87,7 @@ _SIGS = {
     "mps_validate_csr64": [_p, _p, _p],
 }
 _RESTYPES = {"mps_abi_version": ctypes.c_int, "mps_status_string": ctypes.c_char_p,
-             "mps_last_error": ctypes.c_char_p}
+             "mps_last_error": ctypes.c_char_p, "mps_ipc_handle_bytes": ctypes.c_size_t}
 
 
 def _load():
@@ -93,6 +98,13 @@ def _load():
         except Exception as e:  # no silent fallback: the CUDA path is the product
             raise ImportError("libmpspmm.so is missing and could not be built: %s" % e) from e
     lib = ctypes.CDLL(LIB_PATH)
+    if not all(hasattr(lib, name) for name in _SIGS) and "MPS_LIB" not in os.environ:
+        # a stale in-tree build that predates an entry point: rebuild it once, reload
+        import _ctypes
+        from . import _build
+        _ctypes.dlclose(lib._handle)
+        _build.build(force=True)
+        lib = ctypes.CDLL(LIB_PATH)
     for name, args in _SIGS.items():
         f = getattr(lib, name)
         f.argtypes = args

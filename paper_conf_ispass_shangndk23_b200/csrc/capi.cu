@@ -7,6 +7,8 @@
 #include <type_traits>
 #include <vector>
 
+#include <cuda.h>
+
 #include "mps_internal.cuh"
 
 namespace mps { int num_sms(); }
@@ -830,6 +832,66 @@ mps_status mps_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const v
         return fail(MPS_ERR_UNSUPPORTED, "xw: need 16 <= N <= 256, N %% 16 == 0, ld %% 8 == 0, "
                     "16-B aligned pointers");
     MPS_CUDA(e, "xw gemm");
+    return MPS_OK;
+}
+
+mps_status mps_xw_bf16_bcast(const void *X, int64_t n_rows, int64_t F, int64_t ldx,
+                             const void *Wt, int32_t N, int64_t ldw, void *const *B_dsts_host,
+                             int32_t ndst, int64_t row_offset, int64_t ldb, void *stream) {
+    if (n_rows < 0 || F < 0 || N < 0 || ldx < F || ldw < F || ldb < N || row_offset < 0 ||
+        ndst < 1)
+        return fail(MPS_ERR_INVALID, "bad xw_bcast sizes");
+    if (!B_dsts_host) return fail(MPS_ERR_INVALID, "B_dsts_host NULL");
+    if (n_rows == 0 || N == 0) return MPS_OK;
+    if (!X || !Wt) return fail(MPS_ERR_INVALID, "NULL pointer");
+    const cudaError_t e = mps::launch_xw_bf16_bcast(X, n_rows, F, ldx, Wt, N, ldw, B_dsts_host,
+                                                    ndst, row_offset, ldb, (cudaStream_t)stream);
+    if (e == cudaErrorNotSupported)
+        return fail(MPS_ERR_UNSUPPORTED, "xw_bcast: need 16 <= N <= 256, N %% 16 == 0, ld %% 8 "
+                    "== 0, 16-B aligned non-NULL pointers, 1 <= ndst <= 16");
+    MPS_CUDA(e, "xw gemm bcast");
+    return MPS_OK;
+}
+
+// ---- CUDA IPC: map one rank's device buffer into another rank's address space --------
+size_t mps_ipc_handle_bytes(void) { return sizeof(cudaIpcMemHandle_t); }
+
+mps_status mps_ipc_get_handle(const void *dev_ptr, void *handle_out, int64_t *offset_out) {
+    if (!dev_ptr || !handle_out || !offset_out) return fail(MPS_ERR_INVALID, "NULL pointer");
+    // the handle names the whole allocation; report where dev_ptr sits inside it
+    using RangeFn = CUresult (*)(CUdeviceptr *, size_t *, CUdeviceptr);
+    static RangeFn range = nullptr;
+    if (!range) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &p, cudaEnableDefault, &q) !=
+                cudaSuccess || q != cudaDriverEntryPointSuccess)
+            return fail(MPS_ERR_CUDA, "cuMemGetAddressRange unavailable");
+        range = reinterpret_cast<RangeFn>(p);
+    }
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    if (range(&base, &size, (CUdeviceptr)(uintptr_t)dev_ptr) != CUDA_SUCCESS)
+        return fail(MPS_ERR_INVALID, "not a device allocation");
+    cudaIpcMemHandle_t h;
+    MPS_CUDA(cudaIpcGetMemHandle(&h, (void *)(uintptr_t)base), "cudaIpcGetMemHandle");
+    memcpy(handle_out, &h, sizeof(h));
+    *offset_out = (int64_t)((uintptr_t)dev_ptr - (uintptr_t)base);
+    return MPS_OK;
+}
+
+mps_status mps_ipc_open_handle(const void *handle, void **base_out) {
+    if (!handle || !base_out) return fail(MPS_ERR_INVALID, "NULL pointer");
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle, sizeof(h));
+    MPS_CUDA(cudaIpcOpenMemHandle(base_out, h, cudaIpcMemLazyEnablePeerAccess),
+             "cudaIpcOpenMemHandle");
+    return MPS_OK;
+}
+
+mps_status mps_ipc_close_handle(void *base) {
+    if (!base) return fail(MPS_ERR_INVALID, "NULL pointer");
+    MPS_CUDA(cudaIpcCloseMemHandle(base), "cudaIpcCloseMemHandle");
     return MPS_OK;
 }
 

@@ -85,6 +85,9 @@ cudaError_t launch_hot_columns(const int32_t *col, int64_t nnz, int64_t n, int64
 
 cudaError_t launch_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
                            int32_t N, int64_t ldw, void *Bout, int64_t ldb, cudaStream_t s);
+cudaError_t launch_xw_bf16_bcast(const void *X, int64_t n, int64_t F, int64_t ldx,
+                                 const void *Wt, int32_t N, int64_t ldw, void *const *dsts,
+                                 int32_t nd, int64_t row_offset, int64_t ldb, cudaStream_t s);
 
 int num_sms();
 

@@ -13,6 +13,12 @@
 // The shape is tall and thin (n x F times F x N), so the kernel is HBM-bound on reading X;
 // the tensor cores are far from busy, which is the point: the combination costs one read of
 // X and one write of B.
+//
+// Multi-GPU (NEXT-3, the B replication of the sharder): the same kernel
+// with several destinations.  Rank g computes its row block of B and the epilogue stores
+// every tile into the B replica of EVERY rank (peer HBM over NVLink/NVSwitch, mapped with
+// CUDA IPC), so the all-gather of B is fused into the GEMM that produces it and the NVLink
+// transfer of one tile overlaps the TMA loads and MMAs of the next.
 #include <cuda.h>
 #include <cuda_bf16.h>
 
@@ -25,7 +31,15 @@ namespace {
 constexpr int kXwBM = 128;       // rows of X per CTA (UMMA M)
 constexpr int kXwBK = 64;        // reduction chunk: 64 bf16 = 128 B = one swizzle row
 constexpr int kXwMaxStages = 4;
+constexpr int kXwMaxDst = 16;     // replicas one launch can write (ranks of one NVLink domain)
 constexpr int kXwThreads = 128;
+
+// Destinations of the epilogue: B row (row_offset + r) of each replica.
+struct XwDst {
+    __nv_bfloat16 *p[kXwMaxDst];
+    int nd;
+    int64_t row_offset;
+};
 
 __device__ __forceinline__ uint64_t smem_desc_sw128(uint32_t saddr) {
     // UMMA shared-memory descriptor, K-major, SWIZZLE_128B (cute::UMMA::SmemDescriptor):
@@ -67,8 +81,7 @@ __device__ __forceinline__ void mbar_wait_u32(uint32_t bar, uint32_t parity) {
 
 __global__ void __launch_bounds__(kXwThreads)
 xw_gemm_kernel(const __grid_constant__ CUtensorMap map_x, const __grid_constant__ CUtensorMap map_w,
-               int64_t n, int F, int N, int kXwStages, __nv_bfloat16 *__restrict__ Bout,
-               int64_t ldb) {
+               int64_t n, int F, int N, int kXwStages, const XwDst dst, int64_t ldb) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     // 1024-B aligned carve-up: A stages, B stages, then barriers and the TMEM address
     uint8_t *base = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -173,12 +186,17 @@ xw_gemm_kernel(const __grid_constant__ CUtensorMap map_x, const __grid_constant_
                                                          __uint_as_float(v[2 * i + 1]));
                 pk[i] = *reinterpret_cast<uint32_t *>(&h);
             }
-            uint4 *dst = reinterpret_cast<uint4 *>(Bout + row * ldb + c0);
-            dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-            dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
-            if (cols == 32) {
-                dst[2] = make_uint4(pk[8], pk[9], pk[10], pk[11]);
-                dst[3] = make_uint4(pk[12], pk[13], pk[14], pk[15]);
+            // local replica first, then the peers (rotated by block so that the ranks'
+            // CTAs spread their NVLink stores over all destinations at once)
+            for (int i = 0; i < dst.nd; ++i) {
+                const int d = i == 0 ? 0 : 1 + (int)((blockIdx.x + i - 1) % (dst.nd - 1));
+                uint4 *o = reinterpret_cast<uint4 *>(dst.p[d] + (dst.row_offset + row) * ldb + c0);
+                o[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                o[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+                if (cols == 32) {
+                    o[2] = make_uint4(pk[8], pk[9], pk[10], pk[11]);
+                    o[3] = make_uint4(pk[12], pk[13], pk[14], pk[15]);
+                }
             }
         }
     }
@@ -221,13 +239,22 @@ bool make_map(CUtensorMap *map, const void *ptr, int64_t rows, int64_t cols, int
 
 }  // namespace
 
-// X: bf16 [n][ldx] (F used columns), Wt: bf16 [N][ldw] (= W transposed, F used columns),
-// Bout: bf16 [n][ldb].  Returns cudaErrorNotSupported for shapes the kernel does not cover.
-cudaError_t launch_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
-                           int32_t N, int64_t ldw, void *Bout, int64_t ldb, cudaStream_t s) {
+// X: bf16 [n][ldx] (F used columns), Wt: bf16 [N][ldw] (= W transposed, F used columns);
+// B row (row_offset + r) of every dsts[d] (bf16 [.][ldb]) receives row r of X * W.
+// Returns cudaErrorNotSupported for shapes the kernel does not cover.
+static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
+                             int32_t N, int64_t ldw, void *const *dsts, int nd,
+                             int64_t row_offset, int64_t ldb, cudaStream_t s) {
     if (N < 16 || N > 256 || N % 16 || F < 1 || ldx % 8 || ldw % 8 || ldb % 8 ||
-        ((uintptr_t)X & 15) || ((uintptr_t)Wt & 15) || ((uintptr_t)Bout & 15))
+        ((uintptr_t)X & 15) || ((uintptr_t)Wt & 15) || nd < 1 || nd > kXwMaxDst)
         return cudaErrorNotSupported;
+    XwDst dst{};
+    for (int d = 0; d < nd; ++d) {
+        if (!dsts[d] || ((uintptr_t)dsts[d] & 15)) return cudaErrorNotSupported;
+        dst.p[d] = reinterpret_cast<__nv_bfloat16 *>(dsts[d]);
+    }
+    dst.nd = nd;
+    dst.row_offset = row_offset;
     if (n == 0) return cudaSuccess;
     CUtensorMap mx, mw;
     if (!make_map(&mx, X, n, F, ldx, kXwBM) || !make_map(&mw, Wt, N, F, ldw, N))
@@ -249,9 +276,20 @@ cudaError_t launch_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, con
         attr = true;
     }
     const unsigned grid = (unsigned)((n + kXwBM - 1) / kXwBM);
-    xw_gemm_kernel<<<grid, kXwThreads, smem, s>>>(mx, mw, n, (int)F, N, stages,
-                                                  reinterpret_cast<__nv_bfloat16 *>(Bout), ldb);
+    xw_gemm_kernel<<<grid, kXwThreads, smem, s>>>(mx, mw, n, (int)F, N, stages, dst, ldb);
     return cudaGetLastError();
+}
+
+cudaError_t launch_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
+                           int32_t N, int64_t ldw, void *Bout, int64_t ldb, cudaStream_t s) {
+    void *d[1] = {Bout};
+    return launch_xw(X, n, F, ldx, Wt, N, ldw, d, 1, 0, ldb, s);
+}
+
+cudaError_t launch_xw_bf16_bcast(const void *X, int64_t n, int64_t F, int64_t ldx,
+                                 const void *Wt, int32_t N, int64_t ldw, void *const *dsts,
+                                 int32_t nd, int64_t row_offset, int64_t ldb, cudaStream_t s) {
+    return launch_xw(X, n, F, ldx, Wt, N, ldw, dsts, nd, row_offset, ldb, s);
 }
 
 }  // namespace mps

@@ -122,3 +122,71 @@ class ShardedSpMM:
         self.local(B)
         tails = exchange_tails(self.tail, self.world, self.group)
         return self.settle(tails)
+
+
+# --------------------------------------------------------------------------------
+# NEXT-3 multi-GPU: the combination B = X*W fused with the replication of B
+# --------------------------------------------------------------------------------
+def ipc_handle(t: torch.Tensor):
+    """(handle bytes, byte offset) naming t's device memory for a peer process."""
+    h = ctypes.create_string_buffer(int(L.mps_ipc_handle_bytes()))
+    off = ctypes.c_int64()
+    L.mps_ipc_get_handle(_p(t), h, ctypes.byref(off))
+    return h.raw, off.value
+
+
+class PeerReplicas:
+    """One B replica per rank, every rank holding device pointers to all of them.
+
+    Each rank allocates its own replica (n x N bf16); the CUDA IPC handles are exchanged
+    with an all_gather_object over the process group and the peers' replicas are mapped
+    into this process (peer access over NVLink/NVSwitch).  ``ptrs[0]`` is this rank's own
+    replica, followed by the other ranks' in rank order after it (rank+1, rank+2, ...)."""
+
+    def __init__(self, n: int, N: int, rank: int, world: int, device, group=None):
+        self.n, self.N, self.rank, self.world = n, N, rank, world
+        self.B = torch.empty((n, N), dtype=torch.bfloat16, device=device)
+        self._opened = []
+        mine = ipc_handle(self.B) if world > 1 else (b"", 0)
+        allh = [None] * world
+        if world > 1:
+            dist.all_gather_object(allh, mine, group=group)
+        ptrs = [self.B.data_ptr()]
+        for k in range(1, world):
+            g = (rank + k) % world
+            h, off = allh[g]
+            base = ctypes.c_void_p()
+            L.mps_ipc_open_handle(ctypes.create_string_buffer(h, len(h)), ctypes.byref(base))
+            self._opened.append(base.value)
+            ptrs.append(base.value + off)
+        self.ptrs = ptrs
+
+    def close(self):
+        for b in self._opened:
+            L.mps_ipc_close_handle(ctypes.c_void_p(b))
+        self._opened = []
+
+
+def row_block(n: int, world: int, rank: int):
+    """Rows [r0, r1) of B this rank computes: ceil(n/G) per rank, the last one short."""
+    per = -(-n // world)
+    r0 = min(n, rank * per)
+    return r0, min(n, r0 + per)
+
+
+def xw_replicate(X_rows: torch.Tensor, Wt: torch.Tensor, rep: PeerReplicas, stream=None,
+                 group=None, sync=True):
+    """B = X*W on this rank's row block, written by ONE kernel (mps_xw_bf16_bcast) into
+    every rank's replica.  With sync=True the stream is synchronised and the ranks meet at
+    a barrier, after which every replica holds the whole B."""
+    r0, r1 = row_block(rep.n, rep.world, rep.rank)
+    assert X_rows.shape[0] == r1 - r0 and X_rows.dtype == torch.bfloat16
+    assert Wt.shape[0] == rep.N and Wt.shape[1] == X_rows.shape[1]
+    arr = (ctypes.c_void_p * len(rep.ptrs))(*rep.ptrs)
+    L.mps_xw_bf16_bcast(_p(X_rows), r1 - r0, X_rows.shape[1], X_rows.stride(0), _p(Wt), rep.N,
+                        Wt.stride(0), arr, len(rep.ptrs), r0, rep.B.stride(0), _stream(stream))
+    if sync:
+        (torch.cuda.current_stream() if stream is None else stream).synchronize()
+        if rep.world > 1:
+            dist.barrier(group=group)
+    return rep.B
