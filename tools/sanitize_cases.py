@@ -45,6 +45,47 @@ def run():
     if not np.array_equal(out.astype(np.float64), ref):
         print("MISMATCH shard")
         bad += 1
+    # NEXT-4: int64 row_ptr / nnz coordinates
+    for K in (4, 64, 128):
+        for dt in (torch.float32, torch.bfloat16):
+            m = int(rs.randint(50, 400))
+            rl = rs.randint(0, 20, size=m).astype(np.int32)
+            rl[rs.randint(m)] = 900
+            g = G.random_csr(m, 300, rl, K + 1)
+            A = M.CSR(torch.from_numpy(g.row_ptr.astype(np.int64)).cuda(),
+                      torch.from_numpy(g.col_idx).cuda(), torch.from_numpy(g.val).cuda(), g.n)
+            B = G.dense_int(300, K, seed=K)
+            ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+            for fixup in ("atomic", "carry"):
+                for cost in (7, 2048):
+                    C = M.spmm(A, torch.from_numpy(B).cuda().to(dt), fixup=fixup,
+                               items_per_part=cost, min_parts=1)
+                    torch.cuda.synchronize()
+                    if not np.array_equal(C.cpu().numpy().astype(np.float64), ref):
+                        print("MISMATCH int64", K, dt, fixup, cost)
+                        bad += 1
+    # NEXT-3: tcgen05 combination, single destination and 3-replica loopback broadcast
+    import ctypes
+    from paper_conf_ispass_shangndk23_b200.api import _p, _stream
+    gen = torch.Generator().manual_seed(0)
+    n, F, N = 777, 72, 64
+    X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
+    W = torch.randint(-1, 2, (F, N), generator=gen).to(torch.bfloat16)
+    ref = X.double() @ W.double()
+    Xd, Wt = X.cuda(), W.t().contiguous().cuda()
+    if not torch.equal(M.xw_bf16(Xd, Wt).double().cpu(), ref):
+        print("MISMATCH xw")
+        bad += 1
+    reps = [torch.zeros((n, N), dtype=torch.bfloat16, device="cuda") for _ in range(3)]
+    for r in range(3):
+        r0, r1 = M.row_block(n, 3, r)
+        arr = (ctypes.c_void_p * 3)(*[reps[(r + k) % 3].data_ptr() for k in range(3)])
+        M.mps_xw_bf16_bcast(_p(Xd[r0:r1]), r1 - r0, F, F, _p(Wt), N, F, arr, 3, r0, N,
+                            _stream())
+    torch.cuda.synchronize()
+    if not all(torch.equal(t.double().cpu(), ref) for t in reps):
+        print("MISMATCH xw bcast")
+        bad += 1
     print("sanitize cases done, mismatches:", bad)
     return bad
 
