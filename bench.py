@@ -52,6 +52,9 @@ def parse():
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N > 1 process-group backend (gloo: CPU-staged tails, for testing "
                          "several ranks on one GPU)")
+    ap.add_argument("--tails", default="auto", choices=["auto", "p2p", "nccl"],
+                    help="N>1 tail exchange: p2p = fused into the final kernel over peer "
+                         "memory (auto: p2p if it sets up and cross-checks, else nccl)")
     ap.add_argument("--hot", default="auto", choices=["auto", "off"],
                     help="degree-aware L2 residency of B rows (auto: when B exceeds L2/2)")
     ap.add_argument("--cuda-graph", action="store_true",
@@ -185,6 +188,15 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def n_tiles(n, K, b_elt, l2):
+    """Column tiles the library runs for K (capi.cu choose_vec with aligned buffers):
+    32 lanes x 16 B x 4 slots per pass, 256-B row slices when B exceeds half the L2."""
+    t = 512 if b_elt == 4 else 1024
+    if n * K * b_elt > 0.5 * l2:
+        t = min(t, 256 // b_elt)
+    return -(-K // min(K, t))
+
+
 # input feature width F of the combination X*W per workload (the datasets' feature sizes;
 # synthetic R-MAT: 64)
 FEATURES = {"cora": 1433, "pubmed": 500, "reddit": 602, "products": 100, "rmat": 64}
@@ -313,7 +325,7 @@ def main():
         nb = ctypes.c_size_t()
         L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt_code, P, fix, ctypes.byref(nb))
         ws = torch.empty(max(nb.value, 1), dtype=torch.uint8, device=dev)
-        tiles = -(-K // 512) if args.dtype == "f32" else -(-K // 1024)
+        tiles = n_tiles(g.n, K, b_elt, l2)
         launches_per_step = 1 + tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1)
         hot_rows = ctypes.c_int64(-1)
         if args.hot == "auto":
@@ -370,16 +382,47 @@ def main():
             except Exception as e:  # pragma: no cover
                 xw_rep = {"error": str(e)[:200]}
             dist.barrier()
-        sh = M.ShardedSpMM(g.row_ptr, g.col_idx, g.val, g.n, K, rank, world, dev,
-                           b_dtype=tdtype, fixup=args.fixup, items_per_part=args.items_per_part,
-                           min_parts=args.min_parts)
+        sh_kw = dict(b_dtype=tdtype, fixup=args.fixup, items_per_part=args.items_per_part,
+                     min_parts=args.min_parts)
+        tails_mode = "nccl"
+        sh = None
+        if args.tails in ("auto", "p2p") and world <= 16:
+            try:   # mailboxes over CUDA IPC; any failure falls back to the NCCL exchange
+                sh = M.ShardedSpMM(g.row_ptr, g.col_idx, g.val, g.n, K, rank, world, dev,
+                                   tails="p2p", **sh_kw)
+                tails_mode = "p2p"
+            except Exception as e:  # pragma: no cover
+                print("p2p tails unavailable on rank %d: %s" % (rank, e), file=sys.stderr)
+        ok = torch.tensor([1 if tails_mode == "p2p" else 0], device=dev)
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if int(ok[0]) == 1:
+            # cross-check one step of each exchange before trusting the fused one
+            sh.local(Bd)
+            sh.settle(M.exchange_tails(sh.tail, world))
+            ref_rows = sh.C[: sh.rows].clone()
+            sh.local_p2p(Bd)
+            torch.cuda.synchronize(dev)
+            same = torch.allclose(sh.C[: sh.rows], ref_rows, rtol=1e-5, atol=1e-6)
+            ok = torch.tensor([1 if same else 0], device=dev)
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+            del ref_rows
+        if int(ok[0]) != 1:
+            tails_mode = "nccl"
+            if sh is None:
+                sh = M.ShardedSpMM(g.row_ptr, g.col_idx, g.val, g.n, K, rank, world, dev, **sh_kw)
         P, Lp = None, None
-        tiles = -(-K // 512) if args.dtype == "f32" else -(-K // 1024)
-        launches_per_step = 2 + tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1) + 1
+        tiles = n_tiles(g.n, K, b_elt, l2)
+        launches_per_step = 1 + tiles * (2 if fix == L.MPS_FIXUP_CARRY else 1) + \
+            (0 if tails_mode == "p2p" else 1)
 
         def step(ev=None):
             if ev is not None:
                 ev[0].record(stream)
+            if tails_mode == "p2p":       # exchange fused into the final kernel (peer memory)
+                sh.local_p2p(Bd)
+                if ev is not None:
+                    ev[1].record(stream)
+                return
             sh.local(Bd)
             if ev is not None:
                 ev[1].record(stream)
@@ -531,6 +574,7 @@ def main():
                        "read": "flushed before every timed step (2x L2 read, untimed)",
                        "none": "not flushed (col/val > L2)"}[args.flush],
                 "parallelism": "merge-path shards x%d" % world, "graph_sha": g.digest(),
+                "tail_exchange": (tails_mode if world > 1 else None),
                 "cuda_graph": bool(args.cuda_graph and world == 1),
                 "hot_rows": (hot_rows if world == 1 else None),
                 "gen_s": round(gen_s, 2),

@@ -256,6 +256,29 @@ mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int6
                           int64_t ldc, float *tail_out, int32_t fixup, void *workspace,
                           size_t workspace_bytes, void *stream);
 
+/* a6 with the tail exchange over peer memory instead of a collective (fused into the
+ * kernel that finalises the tail: the last column tile's segment kernel in atomic mode,
+ * the carry reduction in carry mode).  The LAST CTA of that kernel
+ *   - pushes this rank's tail (row tail_rows[rank]) into the mailbox of the row's owner
+ *     (owner(r) = max{g : X_g <= r}) and raises flag[rank] there to `epoch`;
+ *   - if other ranks' tails belong to this rank's first row, waits for their flags to
+ *     reach `epoch` and adds them to the row in ascending rank order, then acknowledges.
+ * No mps_apply_tails / all-gather is needed.  mailboxes_host: HOST array of `world`
+ * device pointers, entry g = rank g's mailbox of mps_shard_mailbox_bytes(K) bytes
+ * (this rank's own, peers' mapped with mps_ipc_open_handle); every mailbox must be
+ * zeroed once before the first call.  epoch: 1 for the first call, +1 per call (two
+ * inbox slots alternate; a push waits for the owner's acknowledgement of epoch - 2).
+ * world <= 16.  Waits are bounded (~20 s), after which the kernel traps
+ * (MPS_ERR_CUDA on the next call) rather than hang.  Other arguments: mps_spmm_shard. */
+size_t mps_shard_mailbox_bytes(int32_t K);
+mps_status mps_spmm_shard_p2p(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                              int32_t K, const int32_t *X, const int32_t *Y,
+                              const int32_t *tail_rows, int32_t rank, int32_t world,
+                              int64_t items_per_part, int64_t min_parts, float *C_local,
+                              int64_t ldc, float *tail_out, int32_t fixup,
+                              void *const *mailboxes_host, uint32_t epoch, void *workspace,
+                              size_t workspace_bytes, void *stream);
+
 /* After an all-gather of every rank's tail_out into tails (device float[world*K],
  * rank-major): add the tails whose row this rank owns (owner(r) = max{g : X_g <= r})
  * into C_local, in ascending rank order (deterministic).                         */

@@ -76,6 +76,9 @@ _SIGS = {
     "mps_ipc_get_handle": [_p, _p, _p],
     "mps_ipc_open_handle": [_p, _p],
     "mps_ipc_close_handle": [_p],
+    "mps_shard_mailbox_bytes": [_i32],
+    "mps_spmm_shard_p2p": [_p, _p, _i32, _i64, _i32, _p, _p, _p, _i32, _i32, _i64, _i64, _p,
+                           _i64, _p, _i32, _p, ctypes.c_uint32, _p, _sz, _p],
     "mps_plan64": [_i64, _i64, _i32, _i32, _i64, _i64, _p, _p],
     "mps_partition64": [_p, _i64, _i64, _i64, _i64, _i64, _i64, _p, _p, _p],
     "mps_spmm64_workspace_bytes": [_p, _i32, _i32, _i64, _i32, _p],
@@ -87,7 +90,8 @@ _SIGS = {
     "mps_validate_csr64": [_p, _p, _p],
 }
 _RESTYPES = {"mps_abi_version": ctypes.c_int, "mps_status_string": ctypes.c_char_p,
-             "mps_last_error": ctypes.c_char_p, "mps_ipc_handle_bytes": ctypes.c_size_t}
+             "mps_last_error": ctypes.c_char_p, "mps_ipc_handle_bytes": ctypes.c_size_t,
+             "mps_shard_mailbox_bytes": ctypes.c_size_t}
 
 
 def _load():

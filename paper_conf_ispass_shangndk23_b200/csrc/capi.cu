@@ -206,6 +206,9 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
     const int eb = elt_bytes(dt);
     for (int32_t c0 = 0; c0 < K; c0 += v.tile) {
         mps::SegArgsT<IT> a = base;
+        // the tail exchange rides on the launch that finalises the tail: the last tile's
+        // segment kernel (atomic) or carry reduction (carry)
+        if (c0 + v.tile < K) a.mail.on = 0;
         const int32_t kt = (K - c0) < v.tile ? (K - c0) : v.tile;
         a.K = kt;
         a.B = (const char *)base.B + (size_t)c0 * eb;
@@ -222,7 +225,10 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
         a.l2_hints = hints;
         int V, NR;
         tile_geometry(kt, v.W, &V, &NR);
-        MPS_CUDA(mps::launch_segments(a, dt, v.W, V, NR, fix, s), "segment kernel");
+        mps::SegArgsT<IT> seg_only = a;
+        seg_only.mail.on = 0;
+        MPS_CUDA(mps::launch_segments(fix == mps::FIX_CARRY ? seg_only : a, dt, v.W, V, NR, fix,
+                                      s), "segment kernel");
         if (fix == mps::FIX_CARRY) MPS_CUDA(mps::launch_carry_reduce(a, s), "carry reduce");
         else if (a.relu) MPS_CUDA(mps::launch_relu_split(a, s), "relu on cut rows");
     }
@@ -961,17 +967,37 @@ mps_status mps_spmm_shard_workspace_bytes(const mps_csr *A, int32_t K, int32_t b
     return MPS_OK;
 }
 
-mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                          int32_t K, const int32_t *X, const int32_t *Y,
-                          const int32_t *tail_rows, int32_t rank, int32_t world,
-                          int64_t items_per_part, int64_t min_parts, float *C_local,
-                          int64_t ldc, float *tail_out, int32_t fixup, void *workspace,
-                          size_t workspace_bytes, void *stream) {
-    mps_status st = check_csr(A);
-    if (st) return st;
+}  // extern "C"
+
+static int32_t owner_of(const int32_t *X, int32_t world, int32_t r) {
+    int32_t owner = 0;
+    for (int32_t g = 0; g < world; ++g)
+        if (X[g] <= r) owner = g;
+    return owner;
+}
+
+static mps_status shard_impl(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, const int32_t *X, const int32_t *Y,
+                             const int32_t *tail_rows, int32_t rank, int32_t world,
+                             int64_t items_per_part, int64_t min_parts, float *C_local,
+                             int64_t ldc, float *tail_out, int32_t fixup,
+                             void *const *mailboxes_host, uint32_t epoch, void *workspace,
+                             size_t workspace_bytes, void *stream) {
+    if (!A) return fail(MPS_ERR_INVALID, "A is NULL");
     if (!X || !Y || !tail_rows || world < 1 || rank < 0 || rank >= world)
         return fail(MPS_ERR_INVALID, "bad shard arguments");
+    // a shard without non-zeros may pass NULL col/val (an empty slice): never read
+    mps_csr Aloc = *A;
+    if (Y[rank + 1] == Y[rank] && A->row_ptr) {
+        if (!Aloc.col_idx) Aloc.col_idx = A->row_ptr;
+        if (!Aloc.val) Aloc.val = (const float *)A->row_ptr;
+    }
+    A = &Aloc;
+    mps_status st = check_csr(A);
+    if (st) return st;
     if ((st = check_dense(B, b_dtype, ldb, K, C_local ? C_local : (float *)B, ldc, A))) return st;
+    if (mailboxes_host && (world > mps::kMailMaxWorld || epoch == 0))
+        return fail(MPS_ERR_UNSUPPORTED, "p2p tails: world <= 16 and epoch >= 1");
     if (K == 0) return MPS_OK;
     if (!tail_out) return fail(MPS_ERR_INVALID, "tail_out NULL");
     cudaStream_t s = (cudaStream_t)stream;
@@ -979,9 +1005,46 @@ mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int6
     int64_t P, L, D0, span;
     if ((st = shard_plan(A, X, Y, rank, K, b_dtype, items_per_part, min_parts, &P, &L, &D0, &span)))
         return st;
-    if (span == 0) return MPS_OK;
+    // a6 peer-memory tail exchange: who this rank pushes to and who pushes to it
+    mps::TailMail mail{};
+    if (mailboxes_host && world > 1) {
+        for (int32_t g = 0; g < world; ++g)
+            if (!mailboxes_host[g]) return fail(MPS_ERR_INVALID, "mailbox %d NULL", g);
+        char *mine = (char *)mailboxes_host[rank];
+        const size_t slot = epoch & 1u;
+        mail.counter = (uint32_t *)mine;
+        mail.epoch = epoch;
+        mail.K = K;
+        const int32_t trow = tail_rows[rank];
+        if (trow >= 0) {
+            const int32_t h = owner_of(X, world, trow);
+            char *theirs = (char *)mailboxes_host[h];
+            mail.tail = tail_out;
+            mail.push_dst = (float *)(theirs + mps::kMailInboxOfs) +
+                            (slot * mps::kMailMaxWorld + (size_t)rank) * K;
+            mail.push_flag = (uint32_t *)(theirs + mps::kMailFlagsOfs) + rank;
+            mail.push_ack = (const uint32_t *)(mine + mps::kMailAcksOfs) + h;
+        }
+        for (int32_t g = 0; g < world; ++g) {
+            const int32_t r = tail_rows[g];
+            if (g == rank || r < 0 || owner_of(X, world, r) != rank) continue;
+            mail.pull_mask |= 1u << g;
+            mail.pull_row = C_local + (int64_t)(r - X[rank]) * ldc;
+            mail.ack_dst[g] = (uint32_t *)((char *)mailboxes_host[g] + mps::kMailAcksOfs) + rank;
+        }
+        mail.pull_src = (const float *)(mine + mps::kMailInboxOfs) + slot * mps::kMailMaxWorld * K;
+        mail.pull_flags = (const uint32_t *)(mine + mps::kMailFlagsOfs);
+        mail.on = (mail.push_dst || mail.pull_mask) ? 1 : 0;
+        if (mail.pull_mask && !C_local) return fail(MPS_ERR_INVALID, "C_local NULL");
+    }
     const int fix = resolve_fix(fixup);
     const Vec v = choose_vec(K, b_dtype, B, ldb, C_local ? C_local : tail_out, ldc, A->n);
+    if (span == 0) {
+        // an empty shard still takes part in the exchange: run the final kernel empty
+        if (!mail.on) return MPS_OK;
+        P = 1;
+        L = 0;
+    }
     const size_t need = online_bytes(P, K, v, fix);
     if (!workspace || workspace_bytes < need)
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
@@ -1010,7 +1073,39 @@ mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int6
     a.tail_row = trow;
     a.tail = tail_out;
     a.nnz_end = Y[rank + 1];
+    a.mail = mail;
     return run_segments(a, b_dtype, K, v, fix, rec, s);
+}
+
+extern "C" {
+
+mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                          int32_t K, const int32_t *X, const int32_t *Y,
+                          const int32_t *tail_rows, int32_t rank, int32_t world,
+                          int64_t items_per_part, int64_t min_parts, float *C_local,
+                          int64_t ldc, float *tail_out, int32_t fixup, void *workspace,
+                          size_t workspace_bytes, void *stream) {
+    return shard_impl(A, B, b_dtype, ldb, K, X, Y, tail_rows, rank, world, items_per_part,
+                      min_parts, C_local, ldc, tail_out, fixup, nullptr, 0, workspace,
+                      workspace_bytes, stream);
+}
+
+size_t mps_shard_mailbox_bytes(int32_t K) {
+    return align_up((size_t)mps::kMailInboxOfs +
+                        2 * (size_t)mps::kMailMaxWorld * (size_t)(K > 0 ? K : 0) * 4, 256);
+}
+
+mps_status mps_spmm_shard_p2p(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                              int32_t K, const int32_t *X, const int32_t *Y,
+                              const int32_t *tail_rows, int32_t rank, int32_t world,
+                              int64_t items_per_part, int64_t min_parts, float *C_local,
+                              int64_t ldc, float *tail_out, int32_t fixup,
+                              void *const *mailboxes_host, uint32_t epoch, void *workspace,
+                              size_t workspace_bytes, void *stream) {
+    if (!mailboxes_host) return fail(MPS_ERR_INVALID, "mailboxes_host NULL");
+    return shard_impl(A, B, b_dtype, ldb, K, X, Y, tail_rows, rank, world, items_per_part,
+                      min_parts, C_local, ldc, tail_out, fixup, mailboxes_host, epoch,
+                      workspace, workspace_bytes, stream);
 }
 
 mps_status mps_apply_tails(const float *tails, const int32_t *X, const int32_t *tail_rows,

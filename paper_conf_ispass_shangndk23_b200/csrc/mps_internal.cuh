@@ -16,6 +16,33 @@ constexpr int kBlock = 256;  // threads per CTA for every kernel of the library
 
 enum Fix : int { FIX_ATOMIC = 1, FIX_CARRY = 2 };
 
+// a6 tail exchange over peer memory (NEXT: fused collective).  The last CTA of the kernel
+// that finalises this rank's tail (segment kernel in atomic mode, carry reduce in carry
+// mode; the last column tile) pushes the tail into its owner's mailbox and pulls the tails
+// other ranks pushed for this rank's first row.  Mailbox of every rank (device memory,
+// peers map it with CUDA IPC), bytes:
+//   [0,4)     launch counter (local use)        [64,128)  flags[g]: epoch pushed by rank g
+//   [128,192) acks[h]: epoch consumed by owner h [256, ..) inbox f32 [2 slots][16][K]
+constexpr int kMailMaxWorld = 16;
+constexpr int kMailFlagsOfs = 64, kMailAcksOfs = 128, kMailInboxOfs = 256;
+struct TailMail {
+    uint32_t *counter;          // this rank's launch counter (zeroed between launches)
+    // push (this rank has a tail row owned by another rank)
+    const float *tail;          // the finished local tail, K floats
+    float *push_dst;            // owner's inbox[slot][rank]
+    uint32_t *push_flag;        // owner's flags[rank]
+    const uint32_t *push_ack;   // this rank's acks[owner]
+    // pull (rows of this rank receive tails)
+    float *pull_row;            // this rank's C row that the tails belong to
+    const float *pull_src;      // this rank's inbox[slot]
+    const uint32_t *pull_flags; // this rank's flags
+    uint32_t *ack_dst[kMailMaxWorld];  // sender g's acks[rank]
+    uint32_t pull_mask;         // bit g: rank g pushes a tail to this rank
+    uint32_t epoch;             // >= 1, +1 per step
+    int32_t K;
+    int32_t on;                 // 0: no mailbox work in this launch
+};
+
 // Per-launch arguments of the segment kernel (a3 + a4).  Indices are global merge-path
 // coordinates; col/val are pre-offset so that col[j] is global nnz j (shards hold a
 // slice); C row r lives at C + (r - row_base) * ldc; the row `tail_row` (a shard's cut
@@ -47,6 +74,7 @@ struct SegArgsT {
     const uint32_t *hot; // optional bitmap over B rows: 1 = keep in L2 (evict_last), 0 = stream
     int32_t relu;        // epilogue: 1 = C = max(C, 0) (complete rows at the store; cut rows
                          // by launch_relu_split after the atomics, or in the carry reduce)
+    TailMail mail;       // a6 peer-memory tail exchange (mail.on == 0: none)
 };
 using SegArgs = SegArgsT<int32_t>;
 using SegArgs64 = SegArgsT<int64_t>;
@@ -308,5 +336,70 @@ template <> struct CVec<8> {
         atomicAdd(reinterpret_cast<float4 *>(p + 4), make_float4(v[4], v[5], v[6], v[7]));
     }
 };
+
+// ---- a6 peer-memory tail exchange, run by the last CTA of the finalising kernel -------
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(uint32_t *p, uint32_t v) {
+    asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+// bounded wait (about 20 s) so that a peer that never arrives fails loudly, not forever
+__device__ __forceinline__ void wait_geq(const uint32_t *p, uint32_t v) {
+    for (uint32_t it = 0; ld_acquire_sys(p) < v; ++it) {
+        __nanosleep(256);
+        if (it > (80u << 20)) __trap();
+    }
+}
+
+// Every CTA calls this at exit; the last one to arrive does the exchange.
+__device__ __forceinline__ void tail_mail_epilogue(const TailMail &m) {
+    __shared__ uint32_t s_last;
+    __threadfence();                                      // this CTA's tail / row updates
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const uint32_t t = atomicAdd(m.counter, 1u);
+        s_last = (t == gridDim.x - 1) ? 1u : 0u;
+    }
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();                                      // see every CTA's updates
+    if (m.push_dst) {
+        // the owner must have consumed this slot's previous use (epoch - 2)
+        if (threadIdx.x == 0 && m.epoch > 2) wait_geq(m.push_ack, m.epoch - 2);
+        __syncthreads();
+        for (int c = threadIdx.x; c < m.K; c += blockDim.x)
+            m.push_dst[c] = __ldcg(m.tail + c);
+        __threadfence_system();
+        __syncthreads();
+        if (threadIdx.x == 0) st_release_sys(m.push_flag, m.epoch);
+    }
+    if (m.pull_mask) {
+        uint32_t mask = m.pull_mask;
+        while (mask) {                                    // ascending rank order
+            const int g = __ffs(mask) - 1;
+            mask &= mask - 1;
+            if (threadIdx.x == 0) wait_geq(m.pull_flags + g, m.epoch);
+            __syncthreads();
+            const float *src = m.pull_src + (size_t)g * m.K;
+            for (int c = threadIdx.x; c < m.K; c += blockDim.x)
+                m.pull_row[c] = __ldcg(m.pull_row + c) + __ldcg(src + c);
+            __syncthreads();
+        }
+        __threadfence_system();
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t done = m.pull_mask;
+            while (done) {
+                const int g = __ffs(done) - 1;
+                done &= done - 1;
+                st_release_sys(m.ack_dst[g], m.epoch);
+            }
+        }
+    }
+    if (threadIdx.x == 0) *m.counter = 0u;                // ready for the next launch
+}
 
 }  // namespace mps

@@ -428,6 +428,7 @@ segment_kernel(const SegArgsT<IT> a) {
                 write_row(a.rec + (seg * 2 + (single ? 0 : 1)) * (int64_t)a.kpad, false);
         }
     }
+    if (a.mail.on) tail_mail_epilogue(a.mail);   // a6 tail exchange (last CTA, last tile)
 }
 
 template <int W, int V, int NR, typename TB, int FIX, typename IT>

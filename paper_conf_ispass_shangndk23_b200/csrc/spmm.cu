@@ -29,8 +29,7 @@ cudaError_t launch_segments(const SegArgsT<IT> &a, int b_dtype, int W, int V, in
 // start pieces (slot 0) of segments p, p+1, ... that start inside r.  They are summed
 // in segment order (deterministic) and stored -- no zero-initialisation needed.
 template <typename IT>
-__global__ void __launch_bounds__(kBlock)
-carry_reduce_kernel(const SegArgsT<IT> a) {
+__device__ __forceinline__ void carry_one(const SegArgsT<IT> &a) {
     const int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (p > a.P) return;
@@ -83,6 +82,13 @@ carry_reduce_kernel(const SegArgsT<IT> a) {
             for (int k = 0; c + k < a.K; ++k) dst[c + k] = t[k];
         }
     }
+}
+
+template <typename IT>
+__global__ void __launch_bounds__(kBlock)
+carry_reduce_kernel(const SegArgsT<IT> a) {
+    carry_one(a);
+    if (a.mail.on) tail_mail_epilogue(a.mail);   // a6 tail exchange (carry mode)
 }
 
 template <typename IT>

@@ -72,15 +72,59 @@ def replicate_B(B_rows: torch.Tensor, n: int, world: int, group=None) -> torch.T
     return full[:n]
 
 
+def _open_peers(buf: torch.Tensor, rank: int, world: int, group=None):
+    """All ranks' device pointers to their `buf` (CUDA IPC), indexed by rank, plus the
+    bases this process opened (to close later)."""
+    allh = [None] * world
+    dist.all_gather_object(allh, ipc_handle(buf), group=group)
+    ptrs, opened = [], []
+    for g in range(world):
+        if g == rank:
+            ptrs.append(buf.data_ptr())
+            continue
+        h, off = allh[g]
+        base = ctypes.c_void_p()
+        L.mps_ipc_open_handle(ctypes.create_string_buffer(h, len(h)), ctypes.byref(base))
+        opened.append(base.value)
+        ptrs.append(base.value + off)
+    return ptrs, opened
+
+
+class Mailboxes:
+    """The a6 peer-memory tail exchange's mailboxes (mps_shard_mailbox_bytes each): this
+    rank's own, zeroed, and every peer's mapped through CUDA IPC.  ``ptrs`` is indexed
+    by rank.  For loopback use in one process pass ``ptrs`` of local buffers instead."""
+
+    def __init__(self, K: int, rank: int, world: int, device, group=None, ptrs=None):
+        self.buf = torch.zeros(int(L.mps_shard_mailbox_bytes(K)), dtype=torch.uint8,
+                               device=device)
+        self._opened = []
+        if ptrs is not None:
+            self.ptrs = list(ptrs)
+        else:
+            torch.cuda.synchronize(device)
+            self.ptrs, self._opened = _open_peers(self.buf, rank, world, group)
+            dist.barrier(group=group)        # every mailbox zeroed before any push
+
+    def close(self):
+        for b in self._opened:
+            L.mps_ipc_close_handle(ctypes.c_void_p(b))
+        self._opened = []
+
+
 class ShardedSpMM:
     """Rank-local state of a merge-path sharded SpMM.
 
     row_ptr/col_idx/val: the global CSR on the host (numpy); every rank computes the
-    same bounds, uploads the full row_ptr and only its own [Y_g, Y_{g+1}) slice."""
+    same bounds, uploads the full row_ptr and only its own [Y_g, Y_{g+1}) slice.
+    tails="nccl": the tail vectors are exchanged by one all-gather (exchange_tails) and
+    settled by mps_apply_tails; tails="p2p": the kernel that finalises the tail pushes it
+    into the owner's mailbox over peer memory and pulls the tails owned by this rank
+    (mps_spmm_shard_p2p) -- no collective, no extra launch."""
 
     def __init__(self, row_ptr, col_idx, val, n_cols, K, rank, world, device,
                  b_dtype=torch.float32, fixup="atomic", items_per_part=0, min_parts=0,
-                 group=None):
+                 group=None, tails="nccl", mailbox_ptrs=None):
         self.rank, self.world, self.group, self.K = rank, world, group, K
         self.device = torch.device(device)
         self.fixup, self.ipp, self.minp = fixup, items_per_part, min_parts
@@ -101,6 +145,24 @@ class ShardedSpMM:
         L.mps_spmm_shard_workspace_bytes(ctypes.byref(self.a), K, dt, _p(self.X), rank, world,
                                          items_per_part, min_parts, _fix(fixup), ctypes.byref(nb))
         self.ws = _ws(nb.value, self.device)
+        self.tails = tails
+        self.epoch = 0
+        self.mail = None
+        if tails == "p2p" and world > 1:
+            self.mail = Mailboxes(K, rank, world, self.device, group, ptrs=mailbox_ptrs)
+            self._mp = (ctypes.c_void_p * world)(*self.mail.ptrs)
+
+    def local_p2p(self, B: torch.Tensor, stream=None):
+        """One step with the peer-memory tail exchange: afterwards this rank's C rows are
+        final once every rank's launch of the same epoch has run."""
+        dt = _dtype_code(B)
+        self.epoch += 1
+        L.mps_spmm_shard_p2p(ctypes.byref(self.a), _p(B), dt, B.stride(0), self.K, _p(self.X),
+                             _p(self.Y), _p(self.T), self.rank, self.world, self.ipp, self.minp,
+                             _p(self.C) if self.rows > 0 else None, self.C.stride(0),
+                             _p(self.tail), _fix(self.fixup), self._mp, self.epoch,
+                             _p(self.ws), self.ws.numel(), _stream(stream))
+        return self.C[: self.rows]
 
     def local(self, B: torch.Tensor, stream=None):
         """a2-a4 on this rank's slice: C rows [X_g, X_{g+1}) and the tail vector."""
@@ -119,6 +181,8 @@ class ShardedSpMM:
         return self.C[: self.rows]
 
     def __call__(self, B: torch.Tensor):
+        if self.mail is not None:
+            return self.local_p2p(B)
         self.local(B)
         tails = exchange_tails(self.tail, self.world, self.group)
         return self.settle(tails)
