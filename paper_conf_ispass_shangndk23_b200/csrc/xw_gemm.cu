@@ -22,6 +22,8 @@
 #include <cuda.h>
 #include <cuda_bf16.h>
 
+#include <cstdlib>
+
 #include "mps_internal.cuh"
 
 namespace mps {
@@ -207,6 +209,229 @@ xw_gemm_kernel(const __grid_constant__ CUtensorMap map_x, const __grid_constant_
                      :: "r"(tmem), "r"(ncols) : "memory");
 }
 
+// ---------------------------------------------------------------------------------
+// Persistent variant, used whenever W fits in shared memory next to the X ring: W is
+// loaded ONCE per CTA and stays resident; X tiles stream through an S-stage TMA ring; two
+// TMEM accumulators (2 x N columns) let the epilogue of tile i overlap the MMAs of tile
+// i+1.  Warp roles (320 threads): warp 0 = TMA producer, warp 1 = MMA issuer, warps 2-9 =
+// epilogue (warp w reads TMEM lanes 32*(w%4)..+31; two warps per lane quarter split the
+// columns).  The epilogue stages each 32x32 bf16 block in shared memory (XOR-swizzled)
+// so that global stores write 64 contiguous bytes per row, 8 rows per instruction.
+// ---------------------------------------------------------------------------------
+constexpr int kXpThreads = 320;       // 2 + 8 epilogue warps (two per TMEM lane quarter)
+constexpr int kXpMaxStages = 8;
+
+__global__ void __launch_bounds__(kXpThreads, 1)
+xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
+                     const __grid_constant__ CUtensorMap map_w, int64_t n, int F, int N,
+                     int stages, const XwDst dst, int64_t ldb, int staged) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *base = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const int nk = (F + kXwBK - 1) / kXwBK;
+    const uint32_t a_bytes = kXwBM * kXwBK * 2;            // 16 KB per X stage
+    const uint32_t wchunk = (uint32_t)N * kXwBK * 2;        // one 64-wide chunk of W
+    uint8_t *sW = base;
+    uint8_t *sA = base + (size_t)nk * wchunk;
+    uint64_t *full = (uint64_t *)(sA + (size_t)stages * a_bytes);
+    uint64_t *empty = full + kXpMaxStages;
+    uint64_t *acc_full = empty + kXpMaxStages;              // [2]
+    uint64_t *acc_empty = acc_full + 2;                     // [2]
+    uint64_t *w_full = acc_empty + 2;
+    uint32_t *tmem_slot = (uint32_t *)(w_full + 1);
+    uint8_t *stg = (uint8_t *)(acc_full + 64);              // 8 warps x 32 rows x 64 B
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t ntiles = (n + kXwBM - 1) / kXwBM;
+    const uint32_t ncols = (2 * N) <= 32 ? 32 : ((2 * N) <= 64 ? 64 : ((2 * N) <= 128 ? 128
+                           : ((2 * N) <= 256 ? 256 : 512)));
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kXpMaxStages; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(&acc_full[a], 1);
+            mbar_init(&acc_empty[a], 8);                    // one arrival per epilogue warp
+        }
+        mbar_init(w_full, 1);
+        asm volatile("prefetch.tensormap [%0];" :: "l"(&map_x) : "memory");
+        asm volatile("prefetch.tensormap [%0];" :: "l"(&map_w) : "memory");
+    }
+    mbar_fence_init();
+    if (warp == 1) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                     :: "r"(smem_u32(tmem_slot)), "r"(ncols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---- TMA producer: W once, then the X ring across this CTA's tiles ----
+            mbar_arrive_expect_tx(w_full, (uint32_t)nk * wchunk);
+            for (int kb = 0; kb < nk; ++kb)
+                tma_load_2d(smem_u32(sW + (size_t)kb * wchunk), &map_w, kb * kXwBK, 0,
+                            smem_u32(w_full));
+            uint32_t it = 0;
+            for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+                for (int kb = 0; kb < nk; ++kb, ++it) {
+                    const uint32_t s = it % (uint32_t)stages;
+                    if (it >= (uint32_t)stages)
+                        mbar_wait_u32(smem_u32(&empty[s]), ((it / stages) - 1) & 1);
+                    mbar_arrive_expect_tx(&full[s], a_bytes);
+                    tma_load_2d(smem_u32(sA + (size_t)s * a_bytes), &map_x, kb * kXwBK,
+                                (int)(t * kXwBM), smem_u32(&full[s]));
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ---- MMA issuer ----
+            const uint32_t idesc = instr_desc_bf16(N);
+            mbar_wait_u32(smem_u32(w_full), 0);
+            uint32_t it = 0, i = 0;
+            for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+                const uint32_t acc = i & 1u, use = i >> 1;
+                if (use > 0) mbar_wait_u32(smem_u32(&acc_empty[acc]), (use - 1) & 1);
+                asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                const uint32_t d = tmem + acc * (uint32_t)N;
+                for (int kb = 0; kb < nk; ++kb, ++it) {
+                    const uint32_t s = it % (uint32_t)stages;
+                    mbar_wait_u32(smem_u32(&full[s]), (it / stages) & 1);
+                    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+                    const uint64_t da = smem_desc_sw128(smem_u32(sA + (size_t)s * a_bytes));
+                    const uint64_t db = smem_desc_sw128(smem_u32(sW + (size_t)kb * wchunk));
+#pragma unroll
+                    for (int k = 0; k < kXwBK / 16; ++k) {
+                        const uint32_t accum = (kb > 0 || k > 0) ? 1u : 0u;
+                        asm volatile(
+                            "{\n\t.reg .pred p;\n\t"
+                            "setp.ne.b32 p, %4, 0;\n\t"
+                            "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
+                            :: "r"(d), "l"(da + (uint64_t)(k * 2)), "l"(db + (uint64_t)(k * 2)),
+                               "r"(idesc), "r"(accum) : "memory");
+                    }
+                    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                                 :: "r"(smem_u32(&empty[s])) : "memory");
+                }
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                             :: "r"(smem_u32(&acc_full[acc])) : "memory");
+            }
+        }
+    } else {
+        // ---- epilogue warps 2..9: TMEM -> registers -> bf16 -> every destination ----
+        // warp w drains TMEM lane quarter w % 4 (the hardware's access rule), columns
+        // chunks of 32 alternating between the two warps of a quarter
+        const int q = warp & 3;                              // TMEM lane quarter
+        const int half = (warp - 2) >> 2;
+        uint8_t *wst = stg + (size_t)(warp - 2) * 32 * 64;  // this warp's staging tile
+        uint32_t i = 0;
+        for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+            const uint32_t acc = i & 1u, use = i >> 1;
+            mbar_wait_u32(smem_u32(&acc_full[acc]), use & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            if (half * 32 >= N) {                            // no columns for this warp
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&acc_empty[acc]);
+                continue;
+            }
+            for (int c0 = half * 32; c0 < N; c0 += 64) {
+                uint32_t v[32];
+                const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + acc * (uint32_t)N +
+                                       (uint32_t)c0;
+                asm volatile(
+                    "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+                    "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+                    "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]),
+                      "=r"(v[6]), "=r"(v[7]), "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]),
+                      "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]), "=r"(v[17]),
+                      "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+                      "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]),
+                      "=r"(v[30]), "=r"(v[31])
+                    : "r"(taddr));
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+                if (c0 + 64 >= N) {
+                    // this warp's part is drained: hand it back to the MMA warp early
+                    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&acc_empty[acc]);
+                }
+                if (!staged) {
+                    if (t * kXwBM + q * 32 + lane < n) {
+                        const int64_t row = t * kXwBM + q * 32 + lane;
+                        const int cols = (N - c0) < 32 ? (N - c0) : 32;
+                        uint32_t pk[16];
+#pragma unroll
+                        for (int j = 0; j < 16; ++j) {
+                            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * j]),
+                                                                     __uint_as_float(v[2 * j + 1]));
+                            pk[j] = *reinterpret_cast<uint32_t *>(&h);
+                        }
+                        for (int e = 0; e < dst.nd; ++e) {
+                            const int dd = e == 0 ? 0 : 1 + (int)((blockIdx.x + e - 1) % (dst.nd - 1));
+                            uint4 *o = reinterpret_cast<uint4 *>(dst.p[dd] + (dst.row_offset + row) * ldb + c0);
+                            o[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                            o[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+                            if (cols == 32) {
+                                o[2] = make_uint4(pk[8], pk[9], pk[10], pk[11]);
+                                o[3] = make_uint4(pk[12], pk[13], pk[14], pk[15]);
+                            }
+                        }
+                    }
+                    continue;
+                }
+                // bf16 row slice (64 B) -> this warp's staging tile, 16-B chunks XOR-swizzled
+                // by (row >> 1) & 3 so that both the row-wise writes and the column-wise
+                // reads below hit 8 distinct 16-B bank groups per 8 lanes
+                uint32_t pk[16];
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * j]),
+                                                             __uint_as_float(v[2 * j + 1]));
+                    pk[j] = *reinterpret_cast<uint32_t *>(&h);
+                }
+                uint4 *myst = reinterpret_cast<uint4 *>(wst) + lane * 4;
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    myst[j ^ ((lane >> 1) & 3)] =
+                        make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+                __syncwarp();
+                // coalesced stores: each instruction writes 8 rows x 64 contiguous bytes
+                const int cols = (N - c0) < 32 ? (N - c0) : 32;   // N % 16 == 0: 16 or 32
+                const int j = lane & 3;
+                if (j * 8 < cols) {
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        const int r = k * 8 + (lane >> 2);
+                        const int64_t grow = t * kXwBM + q * 32 + r;
+                        if (grow < n) {
+                            const uint4 val = reinterpret_cast<const uint4 *>(
+                                wst)[r * 4 + (j ^ ((r >> 1) & 3))];
+                            for (int e = 0; e < dst.nd; ++e) {
+                                const int dd = e == 0 ? 0
+                                               : 1 + (int)((blockIdx.x + e - 1) % (dst.nd - 1));
+                                *reinterpret_cast<uint4 *>(dst.p[dd] + (dst.row_offset + grow) * ldb +
+                                                           c0 + j * 8) = val;
+                            }
+                        }
+                    }
+                }
+                __syncwarp();
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 1)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;"
+                     :: "r"(tmem), "r"(ncols) : "memory");
+}
+
 using EncodeFn = CUresult (*)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
                               const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
                               const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
@@ -259,6 +484,61 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
     CUtensorMap mx, mw;
     if (!make_map(&mx, X, n, F, ldx, kXwBM) || !make_map(&mw, Wt, N, F, ldw, N))
         return cudaErrorNotSupported;
+    // persistent kernel when W stays resident next to a >= 2-stage X ring (MPS_XW_PERSIST=0:
+    // always the one-tile-per-CTA kernel; A/B experiments)
+    static const int persist = [] {
+        const char *e = getenv("MPS_XW_PERSIST");
+        return e ? atoi(e) : 1;
+    }();
+    static const int max_stages = [] {
+        const char *e = getenv("MPS_XW_STAGES");
+        return e ? atoi(e) : kXpMaxStages;
+    }();
+    {
+        const int nkp = (int)((F + kXwBK - 1) / kXwBK);
+        const size_t w_bytes = (size_t)nkp * N * kXwBK * 2;
+        const size_t a_bytes = (size_t)kXwBM * kXwBK * 2;
+        const size_t fixed = 1024 + 1024 + 8 * 32 * 64;    // align, barriers, staging
+        const size_t budget = 227u << 10;
+        if (persist && w_bytes + 2 * a_bytes + fixed <= budget) {
+            // Two CTAs per SM when TMEM (2 x 2N columns <= 512) and shared memory allow
+            // >= 2 X stages each (measured: products F=100 N=128 0.31 -> 0.21 ms), else
+            // one CTA with the deepest ring that fits.
+            const size_t half_budget = (113u << 10);
+            int stages;
+            if (4 * N <= 512 && w_bytes + 2 * a_bytes + fixed <= half_budget)
+                stages = (int)((half_budget - fixed - w_bytes) / a_bytes);
+            else
+                stages = (int)((budget - fixed - w_bytes) / a_bytes);
+            stages = stages > max_stages ? max_stages : stages;
+            stages = stages < 2 ? 2 : stages;
+            const size_t smem = fixed + w_bytes + (size_t)stages * a_bytes;
+            static bool pattr = false;
+            if (!pattr) {
+                cudaError_t e = cudaFuncSetAttribute(xw_persistent_kernel,
+                                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                     (int)budget);
+                if (e != cudaSuccess) return e;
+                pattr = true;
+            }
+            // CTAs per SM: shared memory and TMEM (2 accumulators of N columns each)
+            const int per_smem = (int)((228u << 10) / (smem + 1024));
+            const int tcols = 2 * N <= 32 ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128
+                              : (2 * N <= 256 ? 256 : 512)));
+            int per_sm = per_smem < 512 / tcols ? per_smem : 512 / tcols;
+            per_sm = per_sm < 1 ? 1 : (per_sm > 2 ? 2 : per_sm);
+            const int64_t ntiles = (n + kXwBM - 1) / kXwBM;
+            int64_t grid = (int64_t)num_sms() * per_sm;
+            if (grid > ntiles) grid = ntiles;
+            static const int staged = [] {
+                const char *e = getenv("MPS_XW_STAGED");
+                return e ? atoi(e) : 1;
+            }();
+            xw_persistent_kernel<<<(unsigned)grid, kXpThreads, smem, s>>>(mx, mw, n, (int)F, N,
+                                                                          stages, dst, ldb, staged);
+            return cudaGetLastError();
+        }
+    }
     // stages: enough to cover the reduction, but small enough that >= 2 CTAs share an SM
     // (one CTA's epilogue overlaps another's TMA loads); TMEM: <= 2 x 256 columns per SM.
     const size_t stage_bytes = (size_t)kXwBM * kXwBK * 2 + (size_t)N * kXwBK * 2;
