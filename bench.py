@@ -505,6 +505,39 @@ def main():
         with open(prof) as f:
             traffic = json.load(f).get(key)
 
+    # end to end with the graph resident (offline setting): B host -> device,
+    # online SpMM, C device -> host, through mps_spmm_host_dense (context for e2e below)
+    e2e_res = None
+    if world == 1 and args.e2e_steps > 0:
+        Bh_r = torch.from_numpy(Bh).to(tdtype).pin_memory()
+        Ch_r = torch.empty((g.m, K), dtype=torch.float32).pin_memory()
+        nbr = ctypes.c_size_t()
+        L.mps_spmm_host_dense_workspace_bytes(ctypes.byref(a), K, dt_code, K, K,
+                                              args.items_per_part, args.min_parts, fix,
+                                              ctypes.byref(nbr))
+        wsr = torch.empty(nbr.value, dtype=torch.uint8, device=dev)
+
+        def res_step():
+            L.mps_spmm_host_dense(ctypes.byref(a), _p(Bh_r), dt_code, K, K, _p(Ch_r), K,
+                                  args.items_per_part, args.min_parts, fix, _p(wsr), nbr.value,
+                                  s_ptr)
+        res_step()
+        torch.cuda.synchronize(dev)
+        r_ms = []
+        for _ in range(args.e2e_steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            res_step()
+            e1.record(stream)
+            torch.cuda.synchronize(dev)
+            r_ms.append(e0.elapsed_time(e1))
+        t_res = float(np.mean(r_ms))
+        e2e_res = {"value": flops / (t_res * 1e-3) / 1e9, "unit": "GFLOP/s",
+                   "h2d_bytes_per_step": int(b_elt * g.n * K),
+                   "d2h_bytes_per_step": int(4 * g.m * K), "ms_per_step": t_res,
+                   "path": "mps_spmm_host_dense (A resident on the device; pinned host B -> C)"}
+        del wsr, Bh_r, Ch_r
+
     # end-to-end through the public C ABI on pinned HOST buffers (rank 0 layout, N=1)
     e2e = None
     if world == 1 and args.e2e_steps > 0:
@@ -597,6 +630,7 @@ def main():
                 "in_step": False, "fused_xw": xw_rep} if world > 1 else None),
             "cpu_baseline": cpu,
             "e2e": e2e,
+            "e2e_graph_resident": e2e_res,
             "gpu_launches": int(launches_per_step * args.steps),
             "clocks": clk,
         }

@@ -190,6 +190,20 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
                          int64_t items_per_part, int64_t min_parts, int32_t fixup,
                          void *device_workspace, size_t workspace_bytes, void *stream);
 
+/* End to end with the graph resident and the dense operands on the host (the paper's
+ * offline setting: A -- like its schedule -- stays on the device across
+ * inferences; the features B and the output C move every call).  A: DEVICE CSR;
+ * B_host, C_host: host buffers (pinned for asynchronous copies).  Enqueues H2D of B,
+ * the online path and D2H of C on `stream`; the caller synchronises before reading
+ * C_host.  device_workspace: mps_spmm_host_dense_workspace_bytes(...) bytes.        */
+mps_status mps_spmm_host_dense_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                               int64_t ldb, int64_t ldc, int64_t items_per_part,
+                                               int64_t min_parts, int32_t fixup, size_t *bytes);
+mps_status mps_spmm_host_dense(const mps_csr *A, const void *B_host, int32_t b_dtype,
+                               int64_t ldb, int32_t K, float *C_host, int64_t ldc,
+                               int64_t items_per_part, int64_t min_parts, int32_t fixup,
+                               void *device_workspace, size_t workspace_bytes, void *stream);
+
 /* NEXT-3: the GCN combination B = X * W (A*(X*W) order) on the sm_100
  * tensor cores (tcgen05.mma kind::f16, fp32 accumulation in TMEM, TMA-fed), writing B in
  * bf16 into the row-major layout the SpMM gathers (MPS_DT_BF16, ldb).

@@ -64,6 +64,8 @@ _SIGS = {
     "mps_spmm_host_workspace_bytes": [_p, _i32, _i32, _i64, _i64, _i64, _i64, _i32, _p],
     "mps_spmm_host": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _p, _sz, _p],
     "mps_write_stats": [_p, _p, _p, _i64, _p, _p],
+    "mps_spmm_host_dense_workspace_bytes": [_p, _i32, _i32, _i64, _i64, _i64, _i64, _i32, _p],
+    "mps_spmm_host_dense": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _p, _sz, _p],
     "mps_xw_bf16": [_p, _i64, _i64, _i64, _p, _i32, _i64, _p, _i64, _p],
     "mps_shard_bounds": [_p, _i64, _i64, _i32, _p, _p, _p],
     "mps_spmm_shard_workspace_bytes": [_p, _i32, _i32, _p, _i32, _i32, _i64, _i64, _i32, _p],

@@ -243,6 +243,29 @@ def spmm_host(row_ptr, col_idx, val, n_cols, B_host, C_host=None, items_per_part
     return C_host
 
 
+def spmm_host_dense(A: CSR, B_host: torch.Tensor, C_host=None, items_per_part=0, min_parts=0,
+                    fixup="atomic", stream=None, workspace=None):
+    """End to end with the graph resident on A's device and B / C on the host
+    (mps_spmm_host_dense: H2D of B, online SpMM, D2H of C); synchronises, returns C_host."""
+    K = B_host.shape[1]
+    dt = _dtype_code(B_host)
+    if C_host is None:
+        C_host = torch.empty((A.m, K), dtype=torch.float32, pin_memory=True)
+    a = A.struct()
+    nb = ctypes.c_size_t()
+    L.mps_spmm_host_dense_workspace_bytes(ctypes.byref(a), K, dt, B_host.stride(0),
+                                          C_host.stride(0), items_per_part, min_parts,
+                                          _fix(fixup), ctypes.byref(nb))
+    ws = workspace if workspace is not None and workspace.numel() >= nb.value else \
+        _ws(nb.value, A.device)
+    s = torch.cuda.current_stream() if stream is None else stream
+    L.mps_spmm_host_dense(ctypes.byref(a), _p(B_host), dt, B_host.stride(0), K, _p(C_host),
+                          C_host.stride(0), items_per_part, min_parts, _fix(fixup), _p(ws),
+                          ws.numel(), _stream(s))
+    s.synchronize()
+    return C_host
+
+
 def host_workspace_bytes(row_ptr, col_idx, val, n_cols, B_host, C_host, items_per_part=0,
                          min_parts=0, fixup="atomic"):
     K = B_host.shape[1]

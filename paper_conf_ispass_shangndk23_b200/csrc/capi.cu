@@ -827,6 +827,51 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
     return MPS_OK;
 }
 
+mps_status mps_spmm_host_dense_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
+                                               int64_t ldb, int64_t ldc, int64_t items_per_part,
+                                               int64_t min_parts, int32_t fixup, size_t *bytes) {
+    if (!A || !bytes) return fail(MPS_ERR_INVALID, "NULL pointer");
+    size_t online = 0;
+    mps_status st = mps_spmm_online_workspace_bytes(A, K, b_dtype, items_per_part, min_parts,
+                                                    fixup, &online);
+    if (st) return st;
+    *bytes = align_up((size_t)A->n * (size_t)ldb * elt_bytes(b_dtype), 256) +
+             align_up((size_t)A->m * (size_t)ldc * 4, 256) + online;
+    return MPS_OK;
+}
+
+mps_status mps_spmm_host_dense(const mps_csr *A, const void *B_host, int32_t b_dtype,
+                               int64_t ldb, int32_t K, float *C_host, int64_t ldc,
+                               int64_t items_per_part, int64_t min_parts, int32_t fixup,
+                               void *device_workspace, size_t workspace_bytes, void *stream) {
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if ((st = check_dense(B_host, b_dtype, ldb, K, C_host, ldc, A))) return st;
+    if (K == 0 || A->m == 0) return MPS_OK;
+    size_t need = 0, online = 0;
+    if ((st = mps_spmm_host_dense_workspace_bytes(A, K, b_dtype, ldb, ldc, items_per_part,
+                                                  min_parts, fixup, &need)))
+        return st;
+    if ((st = mps_spmm_online_workspace_bytes(A, K, b_dtype, items_per_part, min_parts, fixup,
+                                              &online)))
+        return st;
+    if (!device_workspace || workspace_bytes < need)
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
+    cudaStream_t s = (cudaStream_t)stream;
+    char *w = (char *)device_workspace;
+    const size_t bbytes = (size_t)A->n * (size_t)ldb * elt_bytes(b_dtype);
+    char *Bd = w;
+    float *Cd = (float *)(w + align_up(bbytes, 256));
+    char *ws = (char *)Cd + align_up((size_t)A->m * (size_t)ldc * 4, 256);
+    if (bbytes) MPS_CUDA(cudaMemcpyAsync(Bd, B_host, bbytes, cudaMemcpyHostToDevice, s), "H2D B");
+    if ((st = mps_spmm_online(A, Bd, b_dtype, ldb, K, Cd, ldc, items_per_part, min_parts, fixup,
+                              ws, online, stream)))
+        return st;
+    MPS_CUDA(cudaMemcpyAsync(C_host, Cd, (size_t)A->m * (size_t)ldc * 4, cudaMemcpyDeviceToHost,
+                             s), "D2H C");
+    return MPS_OK;
+}
+
 mps_status mps_xw_bf16(const void *X, int64_t n, int64_t F, int64_t ldx, const void *Wt,
                        int32_t N, int64_t ldw, void *B, int64_t ldb, void *stream) {
     if (n < 0 || F < 0 || N < 0 || ldx < F || ldw < F || ldb < N)

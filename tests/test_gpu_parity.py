@@ -443,6 +443,23 @@ def test_spmm_host_end_to_end():
     assert O.check(C.numpy(), ref, bnd)["ok"]
 
 
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_spmm_host_dense_graph_resident(fixup):
+    g = G.workload("pubmed")
+    A = dev(g)
+    for K, dt in ((64, torch.float32), (16, torch.bfloat16)):
+        B = G.dense_int(g.n, K, seed=K)
+        Bh = torch.from_numpy(B).to(dt).pin_memory()
+        Ci = M.CSR.from_numpy(g.row_ptr, g.col_idx, G.values_int(g.nnz, 3), g.n)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, G.values_int(g.nnz, 3), B, want_bound=False)
+        C = M.spmm_host_dense(Ci, Bh, fixup=fixup)
+        assert np.array_equal(C.numpy().astype(np.float64), ref)
+    Bf = G.features("pubmed", 64)
+    ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bf)
+    C = M.spmm_host_dense(A, torch.from_numpy(Bf).pin_memory(), fixup=fixup)
+    assert O.check(C.numpy(), ref, bnd)["ok"]
+
+
 # --------------------------------------------------------------------------------
 # a6: sharding, loopback on one GPU (every rank run in turn, tails gathered by copy)
 # --------------------------------------------------------------------------------
