@@ -402,7 +402,9 @@ def main():
             ref_rows = sh.C[: sh.rows].clone()
             sh.local_p2p(Bd)
             torch.cuda.synchronize(dev)
-            same = torch.allclose(sh.C[: sh.rows], ref_rows, rtol=1e-5, atol=1e-6)
+            # the two runs differ only in fp32 atomic order: compare against the scale of C
+            scale = float(ref_rows.abs().max()) if ref_rows.numel() else 0.0
+            same = torch.allclose(sh.C[: sh.rows], ref_rows, rtol=1e-4, atol=1e-5 * scale + 1e-30)
             ok = torch.tensor([1 if same else 0], device=dev)
             dist.all_reduce(ok, op=dist.ReduceOp.MIN)
             del ref_rows
