@@ -338,6 +338,23 @@ mps_status mps_spmm64_online(const mps_csr64 *A, const void *B, int32_t b_dtype,
                              int32_t K, float *C, int64_t ldc, int64_t items_per_part,
                              int64_t min_parts, int32_t fixup, int32_t epilogue,
                              void *workspace, size_t workspace_bytes, void *stream);
+/* a6 sharding with 64-bit indices (NEXT-4 scale-out): Y int64[world+1]; the same
+ * closed form, ownership and tail rules as mps_shard_bounds / mps_spmm_shard(_p2p).
+ * mps_spmm_shard64 takes the peer-memory tail exchange's mailboxes_host/epoch (NULL/0 =
+ * none: exchange the tails with an all-gather and mps_apply_tails instead).          */
+mps_status mps_shard_bounds64(const int64_t *row_ptr_host, int64_t m, int64_t nnz,
+                              int32_t world, int32_t *X, int64_t *Y, int32_t *tail_rows);
+mps_status mps_spmm_shard64_workspace_bytes(const mps_csr64 *A, int32_t K, int32_t b_dtype,
+                                            const int32_t *X, int32_t rank, int32_t world,
+                                            int64_t items_per_part, int64_t min_parts,
+                                            int32_t fixup, size_t *bytes);
+mps_status mps_spmm_shard64(const mps_csr64 *A, const void *B, int32_t b_dtype, int64_t ldb,
+                            int32_t K, const int32_t *X, const int64_t *Y,
+                            const int32_t *tail_rows, int32_t rank, int32_t world,
+                            int64_t items_per_part, int64_t min_parts, float *C_local,
+                            int64_t ldc, float *tail_out, int32_t fixup,
+                            void *const *mailboxes_host, uint32_t epoch, void *workspace,
+                            size_t workspace_bytes, void *stream);
 mps_status mps_write_stats64(const mps_csr64 *A, const int32_t *coord_x, const int64_t *coord_y,
                              int64_t num_parts, int64_t *counts_out, void *stream);
 mps_status mps_validate_csr64(const mps_csr64 *A, int64_t *first_bad_host, void *stream);

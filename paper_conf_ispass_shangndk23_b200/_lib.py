@@ -89,6 +89,10 @@ _SIGS = {
     "mps_spmm64_online": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _i32, _p, _sz,
                           _p],
     "mps_write_stats64": [_p, _p, _p, _i64, _p, _p],
+    "mps_shard_bounds64": [_p, _i64, _i64, _i32, _p, _p, _p],
+    "mps_spmm_shard64_workspace_bytes": [_p, _i32, _i32, _p, _i32, _i32, _i64, _i64, _i32, _p],
+    "mps_spmm_shard64": [_p, _p, _i32, _i64, _i32, _p, _p, _p, _i32, _i32, _i64, _i64, _p,
+                         _i64, _p, _i32, _p, ctypes.c_uint32, _p, _sz, _p],
     "mps_validate_csr64": [_p, _p, _p],
 }
 _RESTYPES = {"mps_abi_version": ctypes.c_int, "mps_status_string": ctypes.c_char_p,

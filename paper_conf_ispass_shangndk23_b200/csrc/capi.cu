@@ -954,10 +954,20 @@ mps_status mps_write_stats(const mps_csr *A, const int32_t *coord_x, const int32
 // ----------------------------------------------------------------------------------
 // sharding (a6)
 // ----------------------------------------------------------------------------------
-mps_status mps_shard_bounds(const int32_t *row_ptr_host, int64_t m, int64_t nnz, int32_t world,
-                            int32_t *X, int32_t *Y, int32_t *tail_rows) {
+}  // extern "C"
+
+// ---------------------------------------------------------------------------------
+// a6 sharding, shared by the int32 (mps_csr) and int64 (mps_csr64, NEXT-4) entry points.
+// IT = row_ptr / Y type.
+// ---------------------------------------------------------------------------------
+template <typename IT>
+static mps_status shard_bounds_impl(const IT *row_ptr_host, int64_t m, int64_t nnz,
+                                    int32_t world, int32_t *X, IT *Y, int32_t *tail_rows) {
     if (m < 0 || nnz < 0 || world < 1) return fail(MPS_ERR_INVALID, "bad shard arguments");
-    if (m + nnz >= kMaxIndex) return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (sizeof(IT) == 4 && m + nnz >= kMaxIndex)
+        return fail(MPS_ERR_UNSUPPORTED, "m + nnz >= 2^31");
+    if (sizeof(IT) == 8 && (m >= kMaxIndex || nnz >= kMaxIndex64))
+        return fail(MPS_ERR_UNSUPPORTED, "m >= 2^31 or nnz >= 2^62");
     if (!row_ptr_host || !X || !Y || !tail_rows) return fail(MPS_ERR_INVALID, "NULL pointer");
     const int64_t M = m + nnz;
     const int64_t per = (M + world - 1) / world;
@@ -966,7 +976,7 @@ mps_status mps_shard_bounds(const int32_t *row_ptr_host, int64_t m, int64_t nnz,
         if (d > M) d = M;
         const int64_t x = host_diag_x(row_ptr_host, m, nnz, d);
         X[g] = (int32_t)x;
-        Y[g] = (int32_t)(d - x);
+        Y[g] = (IT)(d - x);
     }
     for (int32_t g = 0; g < world; ++g) {
         const int32_t r = X[g + 1];
@@ -975,41 +985,72 @@ mps_status mps_shard_bounds(const int32_t *row_ptr_host, int64_t m, int64_t nnz,
     return MPS_OK;
 }
 
-static mps_status shard_plan(const mps_csr *A, const int32_t *X, const int32_t *Y,
-                             int32_t rank, int32_t K, int32_t dt, int64_t ipp, int64_t minp,
-                             int64_t *P, int64_t *L, int64_t *D0, int64_t *span) {
+template <typename CSR>
+static mps_status shard_plan(const CSR *A, const int32_t *X, const idx_t<CSR> *Y, int32_t rank,
+                             int32_t K, int32_t dt, int64_t ipp, int64_t minp, int64_t *P,
+                             int64_t *L, int64_t *D0, int64_t *span) {
     if (ipp == 0) ipp = default_cost(A->m, A->nnz, K, dt);  // the whole graph's row length
-    *D0 = (int64_t)X[rank] + Y[rank];
-    const int64_t D1 = (int64_t)X[rank + 1] + Y[rank + 1];
+    *D0 = (int64_t)X[rank] + (int64_t)Y[rank];
+    const int64_t D1 = (int64_t)X[rank + 1] + (int64_t)Y[rank + 1];
     *span = D1 - *D0;
     if (*span < 0) return fail(MPS_ERR_INVALID, "shard bounds not monotone");
     // local plan over the shard's merge items (items of rows counted as rows here)
-    return mps_plan(*span, 0, K, dt, ipp, minp, P, L);
+    return plan_impl(*span, 0, K, dt, ipp, minp, P, L, sizeof(idx_t<CSR>) == 8);
+}
+
+template <typename CSR>
+static mps_status shard_ws_impl(const CSR *A, int32_t K, int32_t b_dtype, const int32_t *X,
+                                int32_t rank, int32_t world, int64_t items_per_part,
+                                int64_t min_parts, int32_t fixup, size_t *bytes) {
+    mps_status st = check_csr(A, false);
+    if (st) return st;
+    if (!X || !bytes || world < 1 || rank < 0 || rank >= world)
+        return fail(MPS_ERR_INVALID, "bad shard arguments");
+    // Y is not needed for the size: the span is at most ceil(M/world)
+    const int64_t M = A->m + A->nnz;
+    const int64_t span = (M + world - 1) / world;
+    int64_t P, L;
+    const int64_t ipp = items_per_part ? items_per_part : default_cost(A->m, A->nnz, K, b_dtype);
+    if ((st = plan_impl(span, 0, K, b_dtype, ipp, min_parts, &P, &L,
+                        sizeof(idx_t<CSR>) == 8)))
+        return st;
+    Vec vmin;
+    vmin.W = 1;
+    vmin.tile = 128;
+    const Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
+    const int fix = resolve_fix(fixup);
+    const size_t ys = sizeof(idx_t<CSR>);
+    size_t a = online_bytes(P, K, v, fix, 0, ys), b = online_bytes(P, K, vmin, fix, 0, ys);
+    *bytes = a > b ? a : b;
+    return MPS_OK;
+}
+
+extern "C" {
+
+mps_status mps_shard_bounds(const int32_t *row_ptr_host, int64_t m, int64_t nnz, int32_t world,
+                            int32_t *X, int32_t *Y, int32_t *tail_rows) {
+    return shard_bounds_impl(row_ptr_host, m, nnz, world, X, Y, tail_rows);
+}
+
+mps_status mps_shard_bounds64(const int64_t *row_ptr_host, int64_t m, int64_t nnz,
+                              int32_t world, int32_t *X, int64_t *Y, int32_t *tail_rows) {
+    return shard_bounds_impl(row_ptr_host, m, nnz, world, X, Y, tail_rows);
 }
 
 mps_status mps_spmm_shard_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
                                           const int32_t *X, int32_t rank, int32_t world,
                                           int64_t items_per_part, int64_t min_parts,
                                           int32_t fixup, size_t *bytes) {
-    mps_status st = check_csr(A, false);
-    if (st) return st;
-    if (!X || !bytes || world < 1 || rank < 0 || rank >= world)
-        return fail(MPS_ERR_INVALID, "bad shard arguments");
-    (void)X;
-    // Y is not needed for the size: the span is at most ceil(M/world)
-    const int64_t M = A->m + A->nnz;
-    const int64_t span = (M + world - 1) / world;
-    int64_t P, L;
-    const int64_t ipp = items_per_part ? items_per_part : default_cost(A->m, A->nnz, K, b_dtype);
-    if ((st = mps_plan(span, 0, K, b_dtype, ipp, min_parts, &P, &L))) return st;
-    Vec vmin;
-    vmin.W = 1;
-    vmin.tile = 128;
-    const Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
-    const int fix = resolve_fix(fixup);
-    size_t a = online_bytes(P, K, v, fix), b = online_bytes(P, K, vmin, fix);
-    *bytes = a > b ? a : b;
-    return MPS_OK;
+    return shard_ws_impl(A, K, b_dtype, X, rank, world, items_per_part, min_parts, fixup,
+                         bytes);
+}
+
+mps_status mps_spmm_shard64_workspace_bytes(const mps_csr64 *A, int32_t K, int32_t b_dtype,
+                                            const int32_t *X, int32_t rank, int32_t world,
+                                            int64_t items_per_part, int64_t min_parts,
+                                            int32_t fixup, size_t *bytes) {
+    return shard_ws_impl(A, K, b_dtype, X, rank, world, items_per_part, min_parts, fixup,
+                         bytes);
 }
 
 }  // extern "C"
@@ -1021,20 +1062,22 @@ static int32_t owner_of(const int32_t *X, int32_t world, int32_t r) {
     return owner;
 }
 
-static mps_status shard_impl(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
-                             int32_t K, const int32_t *X, const int32_t *Y,
+template <typename CSR>
+static mps_status shard_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, const int32_t *X, const idx_t<CSR> *Y,
                              const int32_t *tail_rows, int32_t rank, int32_t world,
                              int64_t items_per_part, int64_t min_parts, float *C_local,
                              int64_t ldc, float *tail_out, int32_t fixup,
                              void *const *mailboxes_host, uint32_t epoch, void *workspace,
                              size_t workspace_bytes, void *stream) {
+    using IT = idx_t<CSR>;
     if (!A) return fail(MPS_ERR_INVALID, "A is NULL");
     if (!X || !Y || !tail_rows || world < 1 || rank < 0 || rank >= world)
         return fail(MPS_ERR_INVALID, "bad shard arguments");
     // a shard without non-zeros may pass NULL col/val (an empty slice): never read
-    mps_csr Aloc = *A;
+    CSR Aloc = *A;
     if (Y[rank + 1] == Y[rank] && A->row_ptr) {
-        if (!Aloc.col_idx) Aloc.col_idx = A->row_ptr;
+        if (!Aloc.col_idx) Aloc.col_idx = (const int32_t *)A->row_ptr;
         if (!Aloc.val) Aloc.val = (const float *)A->row_ptr;
     }
     A = &Aloc;
@@ -1090,18 +1133,20 @@ static mps_status shard_impl(const mps_csr *A, const void *B, int32_t b_dtype, i
         P = 1;
         L = 0;
     }
-    const size_t need = online_bytes(P, K, v, fix);
+    const size_t need = online_bytes(P, K, v, fix, 0, sizeof(IT));
     if (!workspace || workspace_bytes < need)
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
+    const size_t xb = align_up((size_t)(P + 1) * 4, 256);
+    const size_t yb = align_up((size_t)(P + 1) * sizeof(IT), 256);
     int32_t *cx = (int32_t *)workspace;
-    int32_t *cy = (int32_t *)((char *)workspace + align_up((size_t)(P + 1) * 4, 256));
-    void *rec = (char *)workspace + align_up((size_t)(P + 1) * 4, 256) * 2;
+    IT *cy = (IT *)((char *)workspace + xb);
+    void *rec = (char *)workspace + xb + yb;
     const int32_t trow = tail_rows[rank];
-    MPS_CUDA(mps::launch_partition(A->row_ptr, A->m, A->nnz, D0, span, P, L, cx, cy,
-                                   fix == mps::FIX_ATOMIC ? C_local : nullptr, ldc, X[rank], K,
-                                   trow, fix == mps::FIX_ATOMIC ? tail_out : nullptr, s),
+    MPS_CUDA(mps::launch_partition<IT>(A->row_ptr, A->m, A->nnz, D0, span, P, L, cx, cy,
+                                       fix == mps::FIX_ATOMIC ? C_local : nullptr, ldc, X[rank],
+                                       K, trow, fix == mps::FIX_ATOMIC ? tail_out : nullptr, s),
              "partition kernel");
-    mps::SegArgs a{};
+    mps::SegArgsT<IT> a{};
     a.rp = A->row_ptr;
     // col/val hold global nnz [Y[rank], ...): shift so that col[j] is global nnz j
     a.col = (const int32_t *)((uintptr_t)A->col_idx - (uintptr_t)Y[rank] * 4);
@@ -1117,7 +1162,7 @@ static mps_status shard_impl(const mps_csr *A, const void *B, int32_t b_dtype, i
     a.P = P;
     a.tail_row = trow;
     a.tail = tail_out;
-    a.nnz_end = Y[rank + 1];
+    a.nnz_end = (int64_t)Y[rank + 1];
     a.mail = mail;
     return run_segments(a, b_dtype, K, v, fix, rec, s);
 }
@@ -1133,6 +1178,18 @@ mps_status mps_spmm_shard(const mps_csr *A, const void *B, int32_t b_dtype, int6
     return shard_impl(A, B, b_dtype, ldb, K, X, Y, tail_rows, rank, world, items_per_part,
                       min_parts, C_local, ldc, tail_out, fixup, nullptr, 0, workspace,
                       workspace_bytes, stream);
+}
+
+mps_status mps_spmm_shard64(const mps_csr64 *A, const void *B, int32_t b_dtype, int64_t ldb,
+                            int32_t K, const int32_t *X, const int64_t *Y,
+                            const int32_t *tail_rows, int32_t rank, int32_t world,
+                            int64_t items_per_part, int64_t min_parts, float *C_local,
+                            int64_t ldc, float *tail_out, int32_t fixup,
+                            void *const *mailboxes_host, uint32_t epoch, void *workspace,
+                            size_t workspace_bytes, void *stream) {
+    return shard_impl(A, B, b_dtype, ldb, K, X, Y, tail_rows, rank, world, items_per_part,
+                      min_parts, C_local, ldc, tail_out, fixup, mailboxes_host, epoch,
+                      workspace, workspace_bytes, stream);
 }
 
 size_t mps_shard_mailbox_bytes(int32_t K) {

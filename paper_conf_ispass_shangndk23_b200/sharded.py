@@ -21,13 +21,17 @@ from .api import CSR, _p, _stream, _fix, _dtype_code, _ws
 
 
 def shard_bounds(row_ptr_host: np.ndarray, world: int):
-    """Host closed form (mps_shard_bounds): X, Y (int32[world+1]) and tail rows."""
-    rp = np.ascontiguousarray(row_ptr_host, np.int32)
+    """Host closed form (mps_shard_bounds / mps_shard_bounds64 for an int64 row_ptr):
+    X (int32[world+1]), Y (row_ptr's index type, [world+1]) and tail rows."""
+    wide = np.asarray(row_ptr_host).dtype == np.int64
+    it = np.int64 if wide else np.int32
+    rp = np.ascontiguousarray(row_ptr_host, it)
     m, nnz = rp.shape[0] - 1, int(rp[-1])
     X = np.zeros(world + 1, np.int32)
-    Y = np.zeros(world + 1, np.int32)
+    Y = np.zeros(world + 1, it)
     T = np.zeros(world, np.int32)
-    L.mps_shard_bounds(_p(rp), m, nnz, world, _p(X), _p(Y), _p(T))
+    (L.mps_shard_bounds64 if wide else L.mps_shard_bounds)(_p(rp), m, nnz, world, _p(X), _p(Y),
+                                                           _p(T))
     return X, Y, T
 
 
@@ -139,11 +143,14 @@ class ShardedSpMM:
         self.rows = int(self.X[rank + 1]) - self.row0
         self.C = torch.empty((max(self.rows, 1), K), dtype=torch.float32, device=self.device)
         self.tail = torch.zeros(K, dtype=torch.float32, device=self.device)
-        self.a = L.mps_csr(self.m, self.n, self.nnz, _p(self.row_ptr), _p(self.col), _p(self.val))
+        self.wide = self.row_ptr.dtype == torch.int64     # NEXT-4: 64-bit indices
+        cls = L.mps_csr64 if self.wide else L.mps_csr
+        self.a = cls(self.m, self.n, self.nnz, _p(self.row_ptr), _p(self.col), _p(self.val))
         dt = L.MPS_DT_BF16 if b_dtype == torch.bfloat16 else L.MPS_DT_F32
         nb = ctypes.c_size_t()
-        L.mps_spmm_shard_workspace_bytes(ctypes.byref(self.a), K, dt, _p(self.X), rank, world,
-                                         items_per_part, min_parts, _fix(fixup), ctypes.byref(nb))
+        (L.mps_spmm_shard64_workspace_bytes if self.wide else L.mps_spmm_shard_workspace_bytes)(
+            ctypes.byref(self.a), K, dt, _p(self.X), rank, world, items_per_part, min_parts,
+            _fix(fixup), ctypes.byref(nb))
         self.ws = _ws(nb.value, self.device)
         self.tails = tails
         self.epoch = 0
@@ -157,20 +164,24 @@ class ShardedSpMM:
         final once every rank's launch of the same epoch has run."""
         dt = _dtype_code(B)
         self.epoch += 1
-        L.mps_spmm_shard_p2p(ctypes.byref(self.a), _p(B), dt, B.stride(0), self.K, _p(self.X),
-                             _p(self.Y), _p(self.T), self.rank, self.world, self.ipp, self.minp,
-                             _p(self.C) if self.rows > 0 else None, self.C.stride(0),
-                             _p(self.tail), _fix(self.fixup), self._mp, self.epoch,
-                             _p(self.ws), self.ws.numel(), _stream(stream))
+        f = L.mps_spmm_shard64 if self.wide else L.mps_spmm_shard_p2p
+        f(ctypes.byref(self.a), _p(B), dt, B.stride(0), self.K, _p(self.X), _p(self.Y),
+          _p(self.T), self.rank, self.world, self.ipp, self.minp,
+          _p(self.C) if self.rows > 0 else None, self.C.stride(0), _p(self.tail),
+          _fix(self.fixup), self._mp, self.epoch, _p(self.ws), self.ws.numel(), _stream(stream))
         return self.C[: self.rows]
 
     def local(self, B: torch.Tensor, stream=None):
         """a2-a4 on this rank's slice: C rows [X_g, X_{g+1}) and the tail vector."""
         dt = _dtype_code(B)
-        L.mps_spmm_shard(ctypes.byref(self.a), _p(B), dt, B.stride(0), self.K, _p(self.X),
-                         _p(self.Y), _p(self.T), self.rank, self.world, self.ipp, self.minp,
-                         _p(self.C) if self.rows > 0 else None, self.C.stride(0), _p(self.tail),
-                         _fix(self.fixup), _p(self.ws), self.ws.numel(), _stream(stream))
+        args = (ctypes.byref(self.a), _p(B), dt, B.stride(0), self.K, _p(self.X), _p(self.Y),
+                _p(self.T), self.rank, self.world, self.ipp, self.minp,
+                _p(self.C) if self.rows > 0 else None, self.C.stride(0), _p(self.tail),
+                _fix(self.fixup))
+        if self.wide:
+            L.mps_spmm_shard64(*args, None, 0, _p(self.ws), self.ws.numel(), _stream(stream))
+        else:
+            L.mps_spmm_shard(*args, _p(self.ws), self.ws.numel(), _stream(stream))
         return self.C[: self.rows], self.tail
 
     def settle(self, tails_all: torch.Tensor, stream=None):

@@ -98,3 +98,28 @@ def test_plan64_host_only():
     M.mps_spmm64_online_workspace_bytes(ctypes.byref(a), 16, 0, 0, 0, 1, ctypes.byref(nb))
     Pp, Lp = M.plan(1000, 3 * 2 ** 30, 16, 0, 0, 0, wide=True)
     assert nb.value >= (Pp + 1) * 12       # int32 coord_x + int64 coord_y
+
+
+def test_shard_bounds64_host_only():
+    """NEXT-4 scale-out: mps_shard_bounds64 is the Alg. 1 closed form at G diagonals
+    (oracle O4-64 with P = G, L = ceil(M/G)) on a 5e9-non-zero row_ptr; tails by R24."""
+    rs = np.random.RandomState(3)
+    m = 300_000
+    rl = rs.randint(0, 30_000, size=m).astype(np.int64)
+    rl[rs.randint(m, size=2)] = 10 ** 9
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(rl, out=rp[1:])
+    nnz = int(rp[-1])
+    for G_ in (1, 2, 3, 8, 16):
+        X, Y, T = M.shard_bounds(rp, G_)
+        assert Y.dtype == np.int64
+        ox, oy = O.partition64(rp, G_, -(-(m + nnz) // G_))
+        assert np.array_equal(X, ox) and np.array_equal(Y, oy)
+        for g in range(G_):
+            r = X[g + 1]
+            assert T[g] == (r if (r < m and Y[g + 1] > rp[r]) else -1)
+    # the int32 form agrees with the int64 one where both apply
+    g = G.random_csr(500, 300, np.random.RandomState(0).randint(0, 20, 500).astype(np.int32), 1)
+    X32, Y32, T32 = M.shard_bounds(g.row_ptr, 8)
+    X64, Y64, T64 = M.shard_bounds(g.row_ptr.astype(np.int64), 8)
+    assert np.array_equal(X32, X64) and np.array_equal(Y32, Y64) and np.array_equal(T32, T64)

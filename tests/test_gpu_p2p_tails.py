@@ -114,3 +114,35 @@ def test_p2p_tails_two_processes_ipc(tmp_path):
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     oks = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(oks) == 2 and all('"ok": true' in l for l in oks), r.stdout
+
+
+@pytest.mark.parametrize("tails", ["nccl", "p2p"])
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_sharded_int64_loopback(tails, fixup):
+    """NEXT-4 scale-out: sharding with 64-bit indices (mps_spmm_shard64), both exchanges."""
+    world, K = 4, 40
+    for gi, g in enumerate(graphs()):
+        B = G.dense_int(g.n, K, seed=gi)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        Bt = torch.from_numpy(B).cuda()
+        rp64 = g.row_ptr.astype(np.int64)
+        ptrs = None
+        if tails == "p2p":
+            nb = int(M.mps_shard_mailbox_bytes(K))
+            boxes = [torch.zeros(nb, dtype=torch.uint8, device="cuda") for _ in range(world)]
+            ptrs = [b.data_ptr() for b in boxes]
+        sh = [M.ShardedSpMM(rp64, g.col_idx, g.val, g.n, K, r, world, "cuda", fixup=fixup,
+                            items_per_part=9, min_parts=1, tails=tails, mailbox_ptrs=ptrs)
+              for r in range(world)]
+        assert all(s.wide for s in sh)
+        for step in range(2):
+            if tails == "p2p":
+                outs = [s.local_p2p(Bt) for s in sh]
+            else:
+                for s in sh:
+                    s.local(Bt)
+                allt = torch.cat([s.tail for s in sh])
+                outs = [s.settle(allt) for s in sh]
+            torch.cuda.synchronize()
+            C = np.concatenate([o.cpu().numpy() for o in outs])
+            assert np.array_equal(C.astype(np.float64), ref), (gi, step)
