@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="N > 1 process-group backend (gloo: CPU-staged tails, for testing "
                          "several ranks on one GPU)")
+    ap.add_argument("--no-cusparse", action="store_true",
+                    help="skip the cuSPARSE reference point (N=1, fp32)")
     ap.add_argument("--tails", default="auto", choices=["auto", "p2p", "nccl"],
                     help="N>1 tail exchange: p2p = fused into the final kernel over peer "
                          "memory (auto: p2p if it sets up and cross-checks, else nccl)")
@@ -507,6 +509,34 @@ def main():
         with open(prof) as f:
             traffic = json.load(f).get(key)
 
+    # cuSPARSE on the same A, B (reference point; not the product)
+    cus = None
+    if world == 1 and args.dtype == "f32" and not args.no_cusparse:
+        try:
+            import __graft_entry__
+            cl = ctypes.CDLL(__graft_entry__.build_cusparse_ref())
+            bm, ba = ctypes.c_float(), ctypes.c_int()
+            per = (ctypes.c_float * 4)()
+            Cc = torch.empty((g.m, K), dtype=torch.float32, device=dev)
+            rc = cl.cusparse_spmm_best(ctypes.c_int64(g.m), ctypes.c_int64(g.n),
+                                       ctypes.c_int64(g.nnz), _p(A.row_ptr), _p(A.col_idx),
+                                       _p(A.val), _p(Bd), ctypes.c_int64(K), ctypes.c_int32(K),
+                                       _p(Cc), ctypes.c_int64(K), ctypes.c_int(5),
+                                       ctypes.byref(bm), ctypes.byref(ba), per)
+            torch.cuda.synchronize(dev)
+            if rc == 0:
+                names = ["ALG_DEFAULT", "CSR_ALG1", "CSR_ALG2", "CSR_ALG3"]
+                cus = {"ms": bm.value, "gflops": 2.0 * g.nnz * K / (bm.value * 1e-3) / 1e9,
+                       "best_alg": names[ba.value],
+                       "ms_per_alg": {names[i]: (round(per[i], 4) if per[i] >= 0 else None)
+                                      for i in range(4)},
+                       "l2": "flushed before every call", "note": "library SpMM, context only"}
+            else:
+                cus = {"error": "cusparse rc %d" % rc}
+            del Cc
+        except Exception as e:  # pragma: no cover
+            cus = {"error": str(e)[:200]}
+
     # end to end with the graph resident (offline setting): B host -> device,
     # online SpMM, C device -> host, through mps_spmm_host_dense (context for e2e below)
     e2e_res = None
@@ -633,6 +663,7 @@ def main():
             "cpu_baseline": cpu,
             "e2e": e2e,
             "e2e_graph_resident": e2e_res,
+            "cusparse": cus,
             "gpu_launches": int(launches_per_step * args.steps),
             "clocks": clk,
         }
