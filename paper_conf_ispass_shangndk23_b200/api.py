@@ -213,6 +213,15 @@ def xw_bf16(X: torch.Tensor, Wt: torch.Tensor, out: torch.Tensor | None = None, 
     assert X.dtype == torch.bfloat16 and Wt.dtype == torch.bfloat16
     assert X.stride(1) == 1 and Wt.stride(1) == 1 and X.shape[1] == Wt.shape[1]
     n, F = X.shape
+
+    def tma_ready(t):
+        # TMA wants 16-B aligned rows: row stride % 8 bf16 and a 16-B aligned base
+        if t.stride(0) % 8 == 0 and t.data_ptr() % 16 == 0:
+            return t
+        buf = torch.zeros((t.shape[0], -(-t.shape[1] // 8) * 8), dtype=t.dtype, device=t.device)
+        buf[:, : t.shape[1]] = t
+        return buf[:, : t.shape[1]]
+    X, Wt = tma_ready(X), tma_ready(Wt)
     N = Wt.shape[0]
     B = torch.empty((n, N), dtype=torch.bfloat16, device=X.device) if out is None else out
     L.mps_xw_bf16(_p(X), n, F, X.stride(0), _p(Wt), N, Wt.stride(0), _p(B), B.stride(0),

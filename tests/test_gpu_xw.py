@@ -50,3 +50,14 @@ def test_xw_unsupported_shapes_report_errors():
         M.xw_bf16(X, torch.zeros((20, 64), dtype=torch.bfloat16, device="cuda"))   # N % 16
     with pytest.raises(M.MpsError):
         M.xw_bf16(X, torch.zeros((272, 64), dtype=torch.bfloat16, device="cuda"))  # N > 256
+
+
+def test_xw_unaligned_feature_width_is_padded():
+    """F = 1433 (Cora's feature width): rows are not 16-B multiples; the binding pads."""
+    g = torch.Generator(device="cpu").manual_seed(3)
+    X = torch.randint(-1, 2, (500, 1433), generator=g).to(torch.bfloat16)
+    W = torch.randint(-1, 2, (1433, 16), generator=g).to(torch.bfloat16)
+    B = M.xw_bf16(X.cuda(), W.t().contiguous().cuda())
+    ref = X.double() @ W.double()
+    # |sum| <= 1433: bf16 rounds, compare within one bf16 ulp of the exact integer
+    assert torch.all((B.double().cpu() - ref).abs() <= ref.abs() * 2.0 ** -8)
