@@ -226,6 +226,21 @@ mps_status mps_xw_bf16_bcast(const void *X, int64_t n_rows, int64_t F, int64_t l
                              const void *Wt, int32_t N, int64_t ldw, void *const *B_dsts_host,
                              int32_t ndst, int64_t row_offset, int64_t ldb, void *stream);
 
+/* Cross-GPU signals over peer memory, used to pipeline the replication of B (written
+ * tile by tile by mps_xw_bf16_bcast) with the SpMM of the tiles that have arrived.
+ * Signal buffer of every rank: mps_signal_bytes() bytes, zeroed once, flags
+ * [64 slots][16 ranks] uint32.  mps_peer_signal: after everything enqueued earlier on
+ * `stream`, raises flag[slot][rank] to `epoch` in every rank's buffer
+ * (signal_bufs_host: HOST array of `world` device pointers, peers mapped with
+ * mps_ipc_open_handle).  mps_peer_wait: work enqueued after it on `stream` starts once
+ * every rank raised flag[slot][*] to >= epoch in this rank's buffer (bounded wait,
+ * ~20 s, then the kernel traps).  world <= 16, 0 <= slot < 64, epoch >= 1.          */
+size_t mps_signal_bytes(void);
+mps_status mps_peer_signal(void *const *signal_bufs_host, int32_t world, int32_t rank,
+                           int32_t slot, uint32_t epoch, void *stream);
+mps_status mps_peer_wait(const void *my_signal_buf, int32_t world, int32_t slot, uint32_t epoch,
+                         void *stream);
+
 /* CUDA IPC between the ranks of one node (peer access over NVLink is enabled lazily).
  * mps_ipc_get_handle: handle_out (mps_ipc_handle_bytes() bytes, caller-owned) names the
  * device allocation that contains dev_ptr; *offset_out = dev_ptr - its base.  The peer

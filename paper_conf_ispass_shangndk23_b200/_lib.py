@@ -75,6 +75,9 @@ _SIGS = {
     "mps_validate_csr": [_p, _p, _p],
     "mps_xw_bf16_bcast": [_p, _i64, _i64, _i64, _p, _i32, _i64, _p, _i32, _i64, _i64, _p],
     "mps_ipc_handle_bytes": [],
+    "mps_signal_bytes": [],
+    "mps_peer_signal": [_p, _i32, _i32, _i32, ctypes.c_uint32, _p],
+    "mps_peer_wait": [_p, _i32, _i32, ctypes.c_uint32, _p],
     "mps_ipc_get_handle": [_p, _p, _p],
     "mps_ipc_open_handle": [_p, _p],
     "mps_ipc_close_handle": [_p],
@@ -97,7 +100,7 @@ _SIGS = {
 }
 _RESTYPES = {"mps_abi_version": ctypes.c_int, "mps_status_string": ctypes.c_char_p,
              "mps_last_error": ctypes.c_char_p, "mps_ipc_handle_bytes": ctypes.c_size_t,
-             "mps_shard_mailbox_bytes": ctypes.c_size_t}
+             "mps_shard_mailbox_bytes": ctypes.c_size_t, "mps_signal_bytes": ctypes.c_size_t}
 
 
 def _load():

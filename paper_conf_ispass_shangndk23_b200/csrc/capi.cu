@@ -904,6 +904,32 @@ mps_status mps_xw_bf16_bcast(const void *X, int64_t n_rows, int64_t F, int64_t l
     return MPS_OK;
 }
 
+// ---- cross-GPU signals (pipelining the replication of B with the SpMM) ---------------
+constexpr int kSignalSlots = 64;
+size_t mps_signal_bytes(void) { return (size_t)kSignalSlots * mps::kMailMaxWorld * 4; }
+
+mps_status mps_peer_signal(void *const *signal_bufs_host, int32_t world, int32_t rank,
+                           int32_t slot, uint32_t epoch, void *stream) {
+    if (!signal_bufs_host || world < 1 || world > mps::kMailMaxWorld || rank < 0 ||
+        rank >= world || slot < 0 || slot >= kSignalSlots || epoch == 0)
+        return fail(MPS_ERR_INVALID, "bad signal arguments");
+    for (int32_t g = 0; g < world; ++g)
+        if (!signal_bufs_host[g]) return fail(MPS_ERR_INVALID, "signal buffer %d NULL", g);
+    MPS_CUDA(mps::launch_peer_signal(signal_bufs_host, world, rank, slot, epoch,
+                                     (cudaStream_t)stream), "peer signal");
+    return MPS_OK;
+}
+
+mps_status mps_peer_wait(const void *my_signal_buf, int32_t world, int32_t slot, uint32_t epoch,
+                         void *stream) {
+    if (!my_signal_buf || world < 1 || world > mps::kMailMaxWorld || slot < 0 ||
+        slot >= kSignalSlots || epoch == 0)
+        return fail(MPS_ERR_INVALID, "bad wait arguments");
+    MPS_CUDA(mps::launch_peer_wait(my_signal_buf, world, slot, epoch, (cudaStream_t)stream),
+             "peer wait");
+    return MPS_OK;
+}
+
 // ---- CUDA IPC: map one rank's device buffer into another rank's address space --------
 size_t mps_ipc_handle_bytes(void) { return sizeof(cudaIpcMemHandle_t); }
 

@@ -98,6 +98,10 @@ template <typename IT>
 cudaError_t launch_carry_reduce(const SegArgsT<IT> &a, cudaStream_t s);
 template <typename IT>
 cudaError_t launch_relu_split(const SegArgsT<IT> &a, cudaStream_t s);
+cudaError_t launch_peer_signal(void *const *bufs, int world, int rank, int slot, uint32_t epoch,
+                               cudaStream_t s);
+cudaError_t launch_peer_wait(const void *mine, int world, int slot, uint32_t epoch,
+                             cudaStream_t s);
 cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx, int32_t n,
                                float *row, cudaStream_t s);
 template <typename IT>

@@ -149,6 +149,44 @@ cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx
     return cudaGetLastError();
 }
 
+// ---- cross-GPU signals over peer memory (flags[slot][source rank], epoch values) -------
+struct PeerFlags {
+    uint32_t *p[kMailMaxWorld];
+};
+
+// rank `rank` raises flag[slot][rank] to `epoch` in every rank's signal buffer, after
+// everything earlier on this stream (the kernel boundary + a system-scope fence)
+__global__ void peer_signal_kernel(PeerFlags f, int world, int rank, int slot, uint32_t epoch) {
+    const int g = threadIdx.x;
+    __threadfence_system();
+    if (g < world) st_release_sys(f.p[g] + slot * kMailMaxWorld + rank, epoch);
+}
+
+// wait until every rank raised flag[slot][*] to `epoch` in this rank's signal buffer
+__global__ void peer_wait_kernel(const uint32_t *mine, int world, int slot, uint32_t epoch) {
+    const int g = threadIdx.x;
+    if (g < world) wait_geq(mine + slot * kMailMaxWorld + g, epoch);
+    __syncthreads();
+    __threadfence_system();
+}
+
+cudaError_t launch_peer_signal(void *const *bufs, int world, int rank, int slot, uint32_t epoch,
+                               cudaStream_t s) {
+    if (world < 1 || world > kMailMaxWorld) return cudaErrorInvalidValue;
+    PeerFlags f{};
+    for (int g = 0; g < world; ++g) f.p[g] = reinterpret_cast<uint32_t *>(bufs[g]);
+    peer_signal_kernel<<<1, 32, 0, s>>>(f, world, rank, slot, epoch);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_peer_wait(const void *mine, int world, int slot, uint32_t epoch,
+                             cudaStream_t s) {
+    if (world < 1 || world > kMailMaxWorld) return cudaErrorInvalidValue;
+    peer_wait_kernel<<<1, 32, 0, s>>>(reinterpret_cast<const uint32_t *>(mine), world, slot,
+                                      epoch);
+    return cudaGetLastError();
+}
+
 #define MPS_INST_SPMM(IT)                                                                     \
     template cudaError_t launch_segments<IT>(const SegArgsT<IT> &, int, int, int, int, int,     \
                                              cudaStream_t);                                     \

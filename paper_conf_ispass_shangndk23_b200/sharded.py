@@ -159,16 +159,30 @@ class ShardedSpMM:
             self.mail = Mailboxes(K, rank, world, self.device, group, ptrs=mailbox_ptrs)
             self._mp = (ctypes.c_void_p * world)(*self.mail.ptrs)
 
-    def local_p2p(self, B: torch.Tensor, stream=None):
+    def local_p2p(self, B: torch.Tensor, stream=None, c0: int = 0, kt: int | None = None):
         """One step with the peer-memory tail exchange: afterwards this rank's C rows are
-        final once every rank's launch of the same epoch has run."""
+        final once every rank's launch of the same epoch has run.  c0/kt: only columns
+        [c0, c0+kt) of B and C (a column tile; every rank must call the same sequence)."""
         dt = _dtype_code(B)
+        kt = self.K - c0 if kt is None else kt
         self.epoch += 1
+        Bs = B[:, c0:c0 + kt]
+        Cp = self.C[:, c0:] if self.rows > 0 else None
+        if self.mail is None:             # one rank: no tails to exchange
+            assert self.world == 1
+            args = (ctypes.byref(self.a), _p(Bs), dt, B.stride(0), kt, _p(self.X), _p(self.Y),
+                    _p(self.T), 0, 1, self.ipp, self.minp, _p(Cp), self.C.stride(0),
+                    _p(self.tail[c0:]), _fix(self.fixup))
+            if self.wide:
+                L.mps_spmm_shard64(*args, None, 0, _p(self.ws), self.ws.numel(), _stream(stream))
+            else:
+                L.mps_spmm_shard(*args, _p(self.ws), self.ws.numel(), _stream(stream))
+            return self.C[: self.rows]
         f = L.mps_spmm_shard64 if self.wide else L.mps_spmm_shard_p2p
-        f(ctypes.byref(self.a), _p(B), dt, B.stride(0), self.K, _p(self.X), _p(self.Y),
-          _p(self.T), self.rank, self.world, self.ipp, self.minp,
-          _p(self.C) if self.rows > 0 else None, self.C.stride(0), _p(self.tail),
-          _fix(self.fixup), self._mp, self.epoch, _p(self.ws), self.ws.numel(), _stream(stream))
+        f(ctypes.byref(self.a), _p(Bs), dt, B.stride(0), kt, _p(self.X), _p(self.Y),
+          _p(self.T), self.rank, self.world, self.ipp, self.minp, _p(Cp), self.C.stride(0),
+          _p(self.tail[c0:]), _fix(self.fixup), self._mp, self.epoch, _p(self.ws),
+          self.ws.numel(), _stream(stream))
         return self.C[: self.rows]
 
     def local(self, B: torch.Tensor, stream=None):
@@ -265,3 +279,84 @@ def xw_replicate(X_rows: torch.Tensor, Wt: torch.Tensor, rep: PeerReplicas, stre
         if rep.world > 1:
             dist.barrier(group=group)
     return rep.B
+
+
+class ShardedGCNLayer:
+    """One GCN aggregation layer A*(X*W) on G GPUs with the replication of B = X*W
+    pipelined against the SpMM (NEXT-3, multi-GPU).
+
+    Rank g holds rows row_block(n, G, g) of X and the merge-path shard g of A.  B is
+    produced in column tiles of ``tile_cols`` columns; for tile c:
+      stream ``s_xw``:  mps_xw_bf16_bcast writes this rank's rows of B[:, tile c] into
+                        every rank's replica (peer HBM), then mps_peer_signal(slot c);
+      stream ``s_agg``: mps_peer_wait(slot c) -- every rank's rows of tile c arrived --
+                        then the sharded SpMM of tile c with the peer-memory tail exchange.
+    The SpMM of tile c therefore overlaps the GEMM + NVLink transfer of tile c+1.
+    Output: this rank's C rows (fp32, pre-activation).  ``peers``: for loopback use in
+    one process, dict(replicas=[ptr per rank], signals=[ptr per rank],
+    mailboxes=[ptr per rank]); otherwise CUDA IPC over the process group."""
+
+    def __init__(self, row_ptr, col_idx, val, n, F, N, rank, world, device, tile_cols=64,
+                 fixup="atomic", items_per_part=0, min_parts=0, group=None, peers=None):
+        assert N % 16 == 0 and tile_cols % 16 == 0
+        self.n, self.F, self.N, self.rank, self.world = n, F, N, rank, world
+        self.device = torch.device(device)
+        self.tile = min(tile_cols, N)
+        self.tiles = [(c, min(self.tile, N - c)) for c in range(0, N, self.tile)]
+        assert len(self.tiles) <= 64
+        self.sh = ShardedSpMM(row_ptr, col_idx, val, n, N, rank, world, device,
+                              b_dtype=torch.bfloat16, fixup=fixup, items_per_part=items_per_part,
+                              min_parts=min_parts, group=group, tails="p2p",
+                              mailbox_ptrs=None if peers is None else peers["mailboxes"])
+        self.B = torch.empty((n, N), dtype=torch.bfloat16, device=self.device)
+        self.sig = torch.zeros(int(L.mps_signal_bytes()), dtype=torch.uint8, device=self.device)
+        self._opened = []
+        if peers is not None:
+            rep_ptrs, sig_ptrs = list(peers["replicas"]), list(peers["signals"])
+            self.B = peers["B"] if "B" in peers else self.B
+        else:
+            torch.cuda.synchronize(self.device)
+            rep_ptrs, o1 = _open_peers(self.B, rank, world, group)
+            sig_ptrs, o2 = _open_peers(self.sig, rank, world, group)
+            self._opened = o1 + o2
+            dist.barrier(group=group)
+        # destinations for the combination: own replica first, then the others
+        self._dst = [rep_ptrs[(rank + k) % world] for k in range(world)]
+        self._sig = (ctypes.c_void_p * world)(*sig_ptrs)
+        self._mysig = sig_ptrs[rank]
+        self.epoch = 0
+        self.r0, self.r1 = row_block(n, world, rank)
+
+    def replicate(self, X_rows: torch.Tensor, Wt: torch.Tensor, stream):
+        """Enqueue B = X*W tile by tile into every replica, each tile followed by a signal."""
+        self.epoch += 1
+        s = _stream(stream)
+        for slot, (c0, kt) in enumerate(self.tiles):
+            dst = (ctypes.c_void_p * self.world)(*[p + 2 * c0 for p in self._dst])
+            Wc = Wt[c0:c0 + kt]
+            L.mps_xw_bf16_bcast(_p(X_rows), self.r1 - self.r0, X_rows.shape[1], X_rows.stride(0),
+                                _p(Wc), kt, Wt.stride(0), dst, self.world, self.r0, self.N, s)
+            L.mps_peer_signal(self._sig, self.world, self.rank, slot, self.epoch, s)
+
+    def aggregate_tile(self, slot: int, stream):
+        """Enqueue: wait for tile `slot` from every rank, then its sharded SpMM."""
+        c0, kt = self.tiles[slot]
+        L.mps_peer_wait(ctypes.c_void_p(self._mysig), self.world, slot, self.epoch,
+                        _stream(stream))
+        return self.sh.local_p2p(self.B, stream=stream, c0=c0, kt=kt)
+
+    def __call__(self, X_rows: torch.Tensor, Wt: torch.Tensor, s_xw=None, s_agg=None):
+        s_xw = s_xw or torch.cuda.Stream(self.device)
+        s_agg = s_agg or torch.cuda.current_stream(self.device)
+        s_xw.wait_stream(torch.cuda.current_stream(self.device))
+        self.replicate(X_rows, Wt, s_xw)
+        for slot in range(len(self.tiles)):
+            out = self.aggregate_tile(slot, s_agg)
+        return out
+
+    def close(self):
+        for b in self._opened:
+            L.mps_ipc_close_handle(ctypes.c_void_p(b))
+        self._opened = []
+        if self.sh.mail is not None:
+            self.sh.mail.close()

@@ -1,0 +1,114 @@
+"""NEXT-3 multi-GPU: one GCN aggregation layer A*(X*W) with the replication of B = X*W
+pipelined against the sharded SpMM (ShardedGCNLayer: mps_xw_bf16_bcast per column
+tile, mps_peer_signal / mps_peer_wait, mps_spmm_shard_p2p per tile).  Integer-valued X,
+W and A: B is exact in bf16 and C must equal oracle O1 on the fp64 product bit-exactly.
+
+Loopback on one GPU: G ranks' combinations on one stream, then per column tile every
+rank's wait + SpMM in rank order on a second stream (the waits overlap the first)."""
+import numpy as np
+import pytest
+import torch
+
+import graphgen as G
+import oracle as O
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_ispass_shangndk23_b200 as M
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4])
+@pytest.mark.parametrize("N,tile", [(64, 16), (128, 64), (96, 32)])
+def test_sharded_gcn_layer_loopback(world, N, tile):
+    rs = np.random.RandomState(world * 7 + N)
+    n, F = 700, 72
+    rl = rs.randint(0, 12, size=n).astype(np.int32)
+    rl[rs.randint(n)] = 900
+    g = G.random_csr(n, n, rl, 5)
+    gen = torch.Generator().manual_seed(N)
+    X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
+    W = torch.randint(-1, 2, (F, N), generator=gen).to(torch.bfloat16)
+    Bref = (X.double() @ W.double()).numpy()                  # |.| <= 72: exact in bf16
+    ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bref, want_bound=False)
+    Xd, Wt = X.cuda(), W.t().contiguous().cuda()
+    Bs = [torch.full((n, N), float("nan"), dtype=torch.bfloat16, device="cuda")
+          for _ in range(world)]
+    sigs = [torch.zeros(int(M.mps_signal_bytes()), dtype=torch.uint8, device="cuda")
+            for _ in range(world)]
+    boxes = [torch.zeros(int(M.mps_shard_mailbox_bytes(N)), dtype=torch.uint8, device="cuda")
+             for _ in range(world)]
+    layers = []
+    for r in range(world):
+        peers = dict(replicas=[b.data_ptr() for b in Bs], signals=[t.data_ptr() for t in sigs],
+                     mailboxes=[t.data_ptr() for t in boxes], B=Bs[r])
+        layers.append(M.ShardedGCNLayer(g.row_ptr, g.col_idx, g.val, n, F, N, r, world, "cuda",
+                                        tile_cols=tile, items_per_part=23, min_parts=1,
+                                        peers=peers))
+    s_xw, s_agg = torch.cuda.Stream(), torch.cuda.Stream()
+    for step in range(3):                                     # epochs and slots reused
+        for L_ in layers:
+            L_.sh.C.fill_(float("nan"))
+        torch.cuda.synchronize()
+        for L_ in layers:
+            r0, r1 = L_.r0, L_.r1
+            L_.replicate(Xd[r0:r1], Wt, s_xw)
+        for slot in range(len(layers[0].tiles)):
+            for L_ in layers:
+                L_.aggregate_tile(slot, s_agg)
+        torch.cuda.synchronize()
+        for r, L_ in enumerate(layers):
+            assert torch.equal(Bs[r].double().cpu(), torch.from_numpy(Bref)), (step, r)
+        C = np.concatenate([L_.sh.C[: L_.sh.rows].cpu().numpy() for L_ in layers])
+        assert np.array_equal(C.astype(np.float64), ref), step
+
+
+_WORKER = r'''
+import os, sys, json
+sys.path.insert(0, sys.argv[1])
+import numpy as np, torch, torch.distributed as dist
+import graphgen as G, oracle as O
+import paper_conf_ispass_shangndk23_b200 as M
+rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
+torch.cuda.set_device(0)
+dist.init_process_group("gloo")
+n, F, N = 900, 64, 128
+rs = np.random.RandomState(1)
+rl = rs.randint(0, 10, size=n).astype(np.int32); rl[450] = 2000
+g = G.random_csr(n, n, rl, 2)
+gen = torch.Generator().manual_seed(9)
+X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
+W = torch.randint(-1, 2, (F, N), generator=gen).to(torch.bfloat16)
+Bref = (X.double() @ W.double()).numpy()
+ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bref, want_bound=False)
+layer = M.ShardedGCNLayer(g.row_ptr, g.col_idx, g.val, n, F, N, rank, world, "cuda:0",
+                          tile_cols=32, items_per_part=31, min_parts=1)
+r0, r1 = layer.r0, layer.r1
+Xr, Wt = X.cuda()[r0:r1], W.t().contiguous().cuda()
+ok = True
+for step in range(3):
+    torch.cuda.synchronize(); dist.barrier()
+    C = layer(Xr, Wt); torch.cuda.synchronize(); dist.barrier()
+    x0, x1 = int(layer.sh.X[rank]), int(layer.sh.X[rank + 1])
+    ok = ok and np.array_equal(C.cpu().numpy().astype(np.float64), ref[x0:x1])
+layer.close()
+print(json.dumps({"rank": rank, "ok": bool(ok)}))
+dist.destroy_process_group()
+'''
+
+
+def test_sharded_gcn_layer_two_processes_ipc(tmp_path):
+    import os, socket, subprocess, sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    w = tmp_path / "worker.py"
+    w.write_text(_WORKER)
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), str(w), root]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    oks = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(oks) == 2 and all('"ok": true' in l for l in oks), r.stdout
