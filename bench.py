@@ -258,6 +258,49 @@ def xw_replication(M, g, K, rank, world, dev, stream):
             "replicas_equal": bool(t[2] == 0.0)}
 
 
+def gcn_layer_pipelined(M, g, K, rank, world, dev):
+    """NEXT-3 multi-GPU: one aggregation layer A*(X*W) from row-sharded X.  pipelined:
+    ShardedGCNLayer (combination + replication per column tile overlapped with the
+    sharded SpMM of the tiles already resident); serial: the whole replication, a
+    barrier, then the SpMM.  CUDA events, max over ranks, best of 3."""
+    import torch
+    import torch.distributed as dist
+    F = FEATURES.get(g.name.split("-")[0], 64)
+    ldx = -(-F // 8) * 8
+    layer = M.ShardedGCNLayer(g.row_ptr, g.col_idx, g.val, g.n, F, K, rank, world, dev,
+                              tile_cols=64)
+    gen = torch.Generator(device="cpu").manual_seed(1000 + rank)
+    X = torch.zeros((max(layer.r1 - layer.r0, 1), ldx), dtype=torch.bfloat16)
+    X[:, :F] = torch.randn(X.shape[0], F, generator=gen).to(torch.bfloat16)
+    X = X.to(dev)[: layer.r1 - layer.r0, :F]
+    Wt = torch.zeros((K, ldx), dtype=torch.bfloat16)
+    Wt[:, :F] = torch.randn(K, F, generator=torch.Generator().manual_seed(7)) / F ** 0.5
+    Wt = Wt.to(dev)[:, :F]
+    s_xw, s_agg = torch.cuda.Stream(dev), torch.cuda.current_stream(dev)
+    pipe, serial = [], []
+    for _ in range(4):
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s_agg)
+        layer(X, Wt, s_xw=s_xw, s_agg=s_agg)
+        e1.record(s_agg)
+        torch.cuda.synchronize(dev)
+        pipe.append(e0.elapsed_time(e1))
+        dist.barrier()
+        e0.record(s_agg)
+        layer.replicate(X, Wt, s_agg)             # same kernels on one stream: every tile
+        for slot in range(len(layer.tiles)):      # replicated before any SpMM
+            layer.aggregate_tile(slot, s_agg)
+        e1.record(s_agg)
+        torch.cuda.synchronize(dev)
+        serial.append(e0.elapsed_time(e1))
+    t = torch.tensor([min(pipe[1:]), min(serial[1:])], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    layer.close()
+    return {"F": F, "tile_cols": layer.tile, "pipelined_ms": float(t[0]),
+            "serial_ms": float(t[1])}
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -383,6 +426,13 @@ def main():
                 xw_rep = xw_replication(M, g, K, rank, world, dev, stream)
             except Exception as e:  # pragma: no cover
                 xw_rep = {"error": str(e)[:200]}
+            dist.barrier()
+        gcn_layer = None
+        if K % 16 == 0 and 16 <= K <= 256 and world <= 16:
+            try:     # reported beside the step, never allowed to break the bench line
+                gcn_layer = gcn_layer_pipelined(M, g, K, rank, world, dev)
+            except Exception as e:  # pragma: no cover
+                gcn_layer = {"error": str(e)[:200]}
             dist.barrier()
         sh_kw = dict(b_dtype=tdtype, fixup=args.fixup, items_per_part=args.items_per_part,
                      min_parts=args.min_parts)
@@ -659,7 +709,8 @@ def main():
                          "peak_source": peak_src},
             "b_replication": ({"ms": b_rep_ms, "bytes_per_rank_received": int(
                 (world - 1) * (-(-g.n // world)) * K * b_elt), "collective": "all_gather_into_tensor",
-                "in_step": False, "fused_xw": xw_rep} if world > 1 else None),
+                "in_step": False, "fused_xw": xw_rep,
+                "gcn_layer_bf16": gcn_layer} if world > 1 else None),
             "cpu_baseline": cpu,
             "e2e": e2e,
             "e2e_graph_resident": e2e_res,
