@@ -224,7 +224,12 @@ constexpr int kXpMaxStages = 8;
 __global__ void __launch_bounds__(kXpThreads, 1)
 xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
                      const __grid_constant__ CUtensorMap map_w, int64_t n, int F, int N,
-                     int stages, const XwDst dst, int64_t ldb, int staged) {
+                     int stages, const XwDst dst, int64_t ldb, int staged, int nsplit) {
+    // N = the column slice this CTA computes; nsplit slices of W / B are spread over
+    // consecutive CTAs (W too large for shared memory as a whole, or TMEM for 2 CTAs)
+    const int slice = (int)(blockIdx.x % (unsigned)nsplit);
+    const int64_t t0 = blockIdx.x / nsplit, tstride = gridDim.x / nsplit;
+    const int col_off = slice * N;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *base = (uint8_t *)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int nk = (F + kXwBK - 1) / kXwBK;
@@ -274,10 +279,10 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
             // ---- TMA producer: W once, then the X ring across this CTA's tiles ----
             mbar_arrive_expect_tx(w_full, (uint32_t)nk * wchunk);
             for (int kb = 0; kb < nk; ++kb)
-                tma_load_2d(smem_u32(sW + (size_t)kb * wchunk), &map_w, kb * kXwBK, 0,
+                tma_load_2d(smem_u32(sW + (size_t)kb * wchunk), &map_w, kb * kXwBK, col_off,
                             smem_u32(w_full));
             uint32_t it = 0;
-            for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+            for (int64_t t = t0; t < ntiles; t += tstride) {
                 for (int kb = 0; kb < nk; ++kb, ++it) {
                     const uint32_t s = it % (uint32_t)stages;
                     if (it >= (uint32_t)stages)
@@ -294,7 +299,7 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
             const uint32_t idesc = instr_desc_bf16(N);
             mbar_wait_u32(smem_u32(w_full), 0);
             uint32_t it = 0, i = 0;
-            for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+            for (int64_t t = t0; t < ntiles; t += tstride, ++i) {
                 const uint32_t acc = i & 1u, use = i >> 1;
                 if (use > 0) mbar_wait_u32(smem_u32(&acc_empty[acc]), (use - 1) & 1);
                 asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -330,7 +335,7 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
         const int half = (warp - 2) >> 2;
         uint8_t *wst = stg + (size_t)(warp - 2) * 32 * 64;  // this warp's staging tile
         uint32_t i = 0;
-        for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++i) {
+        for (int64_t t = t0; t < ntiles; t += tstride, ++i) {
             const uint32_t acc = i & 1u, use = i >> 1;
             mbar_wait_u32(smem_u32(&acc_full[acc]), use & 1);
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -374,7 +379,8 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
                         }
                         for (int e = 0; e < dst.nd; ++e) {
                             const int dd = e == 0 ? 0 : 1 + (int)((blockIdx.x + e - 1) % (dst.nd - 1));
-                            uint4 *o = reinterpret_cast<uint4 *>(dst.p[dd] + (dst.row_offset + row) * ldb + c0);
+                            uint4 *o = reinterpret_cast<uint4 *>(dst.p[dd] + (dst.row_offset + row) * ldb +
+                                                                 col_off + c0);
                             o[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
                             o[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
                             if (cols == 32) {
@@ -416,7 +422,7 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
                                 const int dd = e == 0 ? 0
                                                : 1 + (int)((blockIdx.x + e - 1) % (dst.nd - 1));
                                 *reinterpret_cast<uint4 *>(dst.p[dd] + (dst.row_offset + grow) * ldb +
-                                                           c0 + j * 8) = val;
+                                                           col_off + c0 + j * 8) = val;
                             }
                         }
                     }
@@ -494,25 +500,41 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
         const char *e = getenv("MPS_XW_STAGES");
         return e ? atoi(e) : kXpMaxStages;
     }();
-    {
+    static const int force_split = [] {
+        const char *e = getenv("MPS_XW_SPLIT");
+        return e ? atoi(e) : 0;
+    }();
+    if (persist) {
+        // Choose the column slice width Nh of W / B one CTA owns (nsplit = N / Nh slices
+        // on consecutive CTAs; X tiles are then read once per slice, the repeats from L2).
+        // Measured (profiles/r01/xw_gemm.md): the whole W (Nh = N) wins whenever it fits,
+        // at two CTAs per SM (TMEM 2 x 2N <= 512 columns, W + >= 2 X stages in half the
+        // shared memory) or else one; slices only when W does not fit at all.
         const int nkp = (int)((F + kXwBK - 1) / kXwBK);
-        const size_t w_bytes = (size_t)nkp * N * kXwBK * 2;
         const size_t a_bytes = (size_t)kXwBM * kXwBK * 2;
-        const size_t fixed = 1024 + 1024 + 8 * 32 * 64;    // align, barriers, staging
-        const size_t budget = 227u << 10;
-        if (persist && w_bytes + 2 * a_bytes + fixed <= budget) {
-            // Two CTAs per SM when TMEM (2 x 2N columns <= 512) and shared memory allow
-            // >= 2 X stages each (measured: products F=100 N=128 0.31 -> 0.21 ms), else
-            // one CTA with the deepest ring that fits.
-            const size_t half_budget = (113u << 10);
-            int stages;
-            if (4 * N <= 512 && w_bytes + 2 * a_bytes + fixed <= half_budget)
-                stages = (int)((half_budget - fixed - w_bytes) / a_bytes);
-            else
-                stages = (int)((budget - fixed - w_bytes) / a_bytes);
+        const size_t fixed = 1024 + 512 + 8 * 32 * 64;      // align, barriers, staging
+        const size_t budget = 227u << 10, half_budget = 113u << 10;
+        auto wb = [&](int nh) { return (size_t)nkp * nh * kXwBK * 2; };
+        int nh = 0, per_sm = 0;
+        for (int d = 1; d <= 4 && nh == 0; d *= 2)
+            for (int pass = 0; pass < 2 && nh == 0; ++pass) {
+                const int c = N / d;
+                if (N % d || c % 16) continue;
+                if (force_split > 0 && d != force_split) continue;
+                if (pass == 0 && 4 * c <= 512 && wb(c) + 2 * a_bytes + fixed <= half_budget) {
+                    nh = c;
+                    per_sm = 2;
+                } else if (pass == 1 && wb(c) + 2 * a_bytes + fixed <= budget) {
+                    nh = c;
+                    per_sm = 1;
+                }
+            }
+        if (nh > 0) {
+            const int nsplit = N / nh;
+            int stages = (int)(((per_sm == 2 ? half_budget : budget) - fixed - wb(nh)) / a_bytes);
             stages = stages > max_stages ? max_stages : stages;
             stages = stages < 2 ? 2 : stages;
-            const size_t smem = fixed + w_bytes + (size_t)stages * a_bytes;
+            const size_t smem = fixed + wb(nh) + (size_t)stages * a_bytes;
             static bool pattr = false;
             if (!pattr) {
                 cudaError_t e = cudaFuncSetAttribute(xw_persistent_kernel,
@@ -521,21 +543,18 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
                 if (e != cudaSuccess) return e;
                 pattr = true;
             }
-            // CTAs per SM: shared memory and TMEM (2 accumulators of N columns each)
-            const int per_smem = (int)((228u << 10) / (smem + 1024));
-            const int tcols = 2 * N <= 32 ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128
-                              : (2 * N <= 256 ? 256 : 512)));
-            int per_sm = per_smem < 512 / tcols ? per_smem : 512 / tcols;
-            per_sm = per_sm < 1 ? 1 : (per_sm > 2 ? 2 : per_sm);
+            CUtensorMap mws;
+            if (nh != N && !make_map(&mws, Wt, N, F, ldw, nh)) return cudaErrorNotSupported;
             const int64_t ntiles = (n + kXwBM - 1) / kXwBM;
-            int64_t grid = (int64_t)num_sms() * per_sm;
-            if (grid > ntiles) grid = ntiles;
+            int64_t grid = (int64_t)num_sms() * per_sm / nsplit * nsplit;
+            if (grid > ntiles * nsplit) grid = ntiles * nsplit;
+            if (grid < nsplit) grid = nsplit;
             static const int staged = [] {
                 const char *e = getenv("MPS_XW_STAGED");
                 return e ? atoi(e) : 1;
             }();
-            xw_persistent_kernel<<<(unsigned)grid, kXpThreads, smem, s>>>(mx, mw, n, (int)F, N,
-                                                                          stages, dst, ldb, staged);
+            xw_persistent_kernel<<<(unsigned)grid, kXpThreads, smem, s>>>(
+                mx, nh == N ? mw : mws, n, (int)F, nh, stages, dst, ldb, staged, nsplit);
             return cudaGetLastError();
         }
     }
