@@ -17,8 +17,11 @@
  *  - Streams: every device call is asynchronous on `stream` (a cudaStream_t passed
  *    as void*; NULL = the legacy default stream).  Only mps_validate_csr
  *    synchronises.
- *  - Index type: int32 row_ptr / col_idx.  M = m + nnz must be < 2^31, else
- *    MPS_ERR_UNSUPPORTED (reading R16).
+ *  - Index type: int32 row_ptr / col_idx through mps_csr (M = m + nnz must be < 2^31,
+ *    else MPS_ERR_UNSUPPORTED, reading R16); int64 row_ptr through mps_csr64 and the
+ *    *64 entry points (NEXT-4).
+ *  - Multi-GPU calls (mps_spmm_shard*, mps_xw_bf16_bcast, mps_peer_*) take peer
+ *    pointers mapped with the mps_ipc_* calls; collectives stay outside the library.
  *  - Errors: MPS_ERR_INVALID for NULL pointers with non-zero sizes, negative sizes,
  *    ldb < K, ldc < K, num_parts < 1, rank outside [0, world); MPS_ERR_UNSUPPORTED
  *    for M >= 2^31 or an unknown dtype; MPS_ERR_WORKSPACE if workspace_bytes is too
