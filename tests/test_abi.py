@@ -123,3 +123,34 @@ def test_shard_bounds64_host_only():
     X32, Y32, T32 = M.shard_bounds(g.row_ptr, 8)
     X64, Y64, T64 = M.shard_bounds(g.row_ptr.astype(np.int64), 8)
     assert np.array_equal(X32, X64) and np.array_equal(Y32, Y64) and np.array_equal(T32, T64)
+
+
+def test_multi_gpu_entry_points_validate_before_touching_the_gpu():
+    """Argument checks of the peer-memory entry points return status codes on a host
+    without a GPU (no device call is reached)."""
+    assert M.mps_signal_bytes() == 64 * 16 * 4
+    assert M.mps_shard_mailbox_bytes(128) >= 256 + 2 * 16 * 128 * 4
+    assert M.mps_shard_mailbox_bytes(128) % 256 == 0
+    arr = (ctypes.c_void_p * 2)(None, None)
+    for call in (lambda: M.mps_peer_signal(None, 2, 0, 0, 1, None),
+                 lambda: M.mps_peer_signal(arr, 2, 0, 0, 1, None),          # NULL buffers
+                 lambda: M.mps_peer_signal(arr, 17, 0, 0, 1, None),         # world > 16
+                 lambda: M.mps_peer_signal(arr, 2, 2, 0, 1, None),          # rank >= world
+                 lambda: M.mps_peer_signal(arr, 2, 0, 64, 1, None),         # slot >= 64
+                 lambda: M.mps_peer_wait(None, 2, 0, 1, None),
+                 lambda: M.mps_peer_wait(ctypes.c_void_p(16), 2, 0, 0, None)):  # epoch 0
+        with pytest.raises(M.MpsError) as e:
+            call()
+        assert e.value.status == M.MPS_ERR_INVALID
+    a = M.mps_csr(10, 10, 0, None, None, None)
+    X = np.zeros(3, np.int32)
+    with pytest.raises(M.MpsError) as e:        # p2p exchange needs the mailbox array
+        M.mps_spmm_shard_p2p(ctypes.byref(a), None, 0, 8, 8, X.ctypes.data_as(ctypes.c_void_p),
+                             X.ctypes.data_as(ctypes.c_void_p), X.ctypes.data_as(ctypes.c_void_p),
+                             0, 2, 0, 0, None, 8, None, 1, None, 1, None, 0, None)
+    assert e.value.status == M.MPS_ERR_INVALID
+    with pytest.raises(M.MpsError) as e:        # more than 16 destinations
+        dst = (ctypes.c_void_p * 17)(*([16] * 17))
+        M.mps_xw_bf16_bcast(ctypes.c_void_p(16), 10, 64, 64, ctypes.c_void_p(16), 32, 64, dst,
+                            17, 0, 32, None)
+    assert e.value.status in (M.MPS_ERR_INVALID, M.MPS_ERR_UNSUPPORTED)
