@@ -229,6 +229,12 @@ mps_status mps_xw_bf16_bcast(const void *X, int64_t n_rows, int64_t F, int64_t l
                              const void *Wt, int32_t N, int64_t ldw, void *const *B_dsts_host,
                              int32_t ndst, int64_t row_offset, int64_t ldb, void *stream);
 
+/* GCN glue between layers (sigma = ReLU): H[r][c] = bf16(max(C[r][c], 0)) for
+ * rows x K (C fp32 with leading dimension ldc, H bf16 with ldh) -- the next layer's
+ * combination input.  Asynchronous on stream.                                        */
+mps_status mps_relu_to_bf16(const float *C, int64_t rows, int32_t K, int64_t ldc, void *H,
+                            int64_t ldh, void *stream);
+
 /* Cross-GPU signals over peer memory, used to pipeline the replication of B (written
  * tile by tile by mps_xw_bf16_bcast) with the SpMM of the tiles that have arrived.
  * Signal buffer of every rank: mps_signal_bytes() bytes, zeroed once, flags

@@ -76,6 +76,7 @@ _SIGS = {
     "mps_xw_bf16_bcast": [_p, _i64, _i64, _i64, _p, _i32, _i64, _p, _i32, _i64, _i64, _p],
     "mps_ipc_handle_bytes": [],
     "mps_signal_bytes": [],
+    "mps_relu_to_bf16": [_p, _i64, _i32, _i64, _p, _i64, _p],
     "mps_peer_signal": [_p, _i32, _i32, _i32, ctypes.c_uint32, _p],
     "mps_peer_wait": [_p, _i32, _i32, ctypes.c_uint32, _p],
     "mps_ipc_get_handle": [_p, _p, _p],

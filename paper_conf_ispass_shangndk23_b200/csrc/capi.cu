@@ -904,6 +904,15 @@ mps_status mps_xw_bf16_bcast(const void *X, int64_t n_rows, int64_t F, int64_t l
     return MPS_OK;
 }
 
+mps_status mps_relu_to_bf16(const float *C, int64_t rows, int32_t K, int64_t ldc, void *H,
+                            int64_t ldh, void *stream) {
+    if (rows < 0 || K < 0 || (rows > 0 && K > 0 && (!C || !H || ldc < K || ldh < K)))
+        return fail(MPS_ERR_INVALID, "bad relu_to_bf16 arguments");
+    MPS_CUDA(mps::launch_relu_to_bf16(C, rows, K, ldc, H, ldh, (cudaStream_t)stream),
+             "relu_to_bf16");
+    return MPS_OK;
+}
+
 // ---- cross-GPU signals (pipelining the replication of B with the SpMM) ---------------
 constexpr int kSignalSlots = 64;
 size_t mps_signal_bytes(void) { return (size_t)kSignalSlots * mps::kMailMaxWorld * 4; }

@@ -102,6 +102,8 @@ cudaError_t launch_peer_signal(void *const *bufs, int world, int rank, int slot,
                                cudaStream_t s);
 cudaError_t launch_peer_wait(const void *mine, int world, int slot, uint32_t epoch,
                              cudaStream_t s);
+cudaError_t launch_relu_to_bf16(const float *C, int64_t rows, int K, int64_t ldc, void *H,
+                                int64_t ldh, cudaStream_t s);
 cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx, int32_t n,
                                float *row, cudaStream_t s);
 template <typename IT>

@@ -149,6 +149,28 @@ cudaError_t launch_apply_tails(const float *tails, int32_t K, const int32_t *idx
     return cudaGetLastError();
 }
 
+// ---- GCN glue: H = bf16(relu(C)), the next layer's combination input ----------------
+__global__ void relu_to_bf16_kernel(const float *__restrict__ C, int64_t rows, int K,
+                                    int64_t ldc, __nv_bfloat16 *__restrict__ H, int64_t ldh) {
+    const int64_t total = rows * (int64_t)K;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = i / K, c = i - r * K;
+        H[r * ldh + c] = __float2bfloat16_rn(fmaxf(__ldg(C + r * ldc + c), 0.f));
+    }
+}
+
+cudaError_t launch_relu_to_bf16(const float *C, int64_t rows, int K, int64_t ldc, void *H,
+                                int64_t ldh, cudaStream_t s) {
+    if (rows <= 0 || K <= 0) return cudaSuccess;
+    int64_t blocks = (rows * K + kBlock - 1) / kBlock;
+    const int64_t cap = (int64_t)num_sms() * 8;
+    if (blocks > cap) blocks = cap;
+    relu_to_bf16_kernel<<<(unsigned)blocks, kBlock, 0, s>>>(
+        C, rows, K, ldc, reinterpret_cast<__nv_bfloat16 *>(H), ldh);
+    return cudaGetLastError();
+}
+
 // ---- cross-GPU signals over peer memory (flags[slot][source rank], epoch values) -------
 struct PeerFlags {
     uint32_t *p[kMailMaxWorld];

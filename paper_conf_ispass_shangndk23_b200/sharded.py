@@ -285,7 +285,8 @@ class ShardedGCNLayer:
     """One GCN aggregation layer A*(X*W) on G GPUs with the replication of B = X*W
     pipelined against the SpMM (NEXT-3, multi-GPU).
 
-    Rank g holds rows row_block(n, G, g) of X and the merge-path shard g of A.  B is
+    Rank g holds the merge-path shard g of A and the rows [X_g, X_{g+1}) of X -- the
+    rows of C it owns, so one layer's output is the next layer's input without moving.  B is
     produced in column tiles of ``tile_cols`` columns; for tile c:
       stream ``s_xw``:  mps_xw_bf16_bcast writes this rank's rows of B[:, tile c] into
                         every rank's replica (peer HBM), then mps_peer_signal(slot c);
@@ -325,7 +326,9 @@ class ShardedGCNLayer:
         self._sig = (ctypes.c_void_p * world)(*sig_ptrs)
         self._mysig = sig_ptrs[rank]
         self.epoch = 0
-        self.r0, self.r1 = row_block(n, world, rank)
+        # the rows of X this rank combines are the rows of C it owns (merge-path shard
+        # rows), so a layer's output rows feed the next layer's combination in place
+        self.r0, self.r1 = int(self.sh.X[rank]), int(self.sh.X[rank + 1])
 
     def replicate(self, X_rows: torch.Tensor, Wt: torch.Tensor, stream):
         """Enqueue B = X*W tile by tile into every replica, each tile followed by a signal."""
@@ -360,3 +363,42 @@ class ShardedGCNLayer:
         self._opened = []
         if self.sh.mail is not None:
             self.sh.mail.close()
+
+
+class ShardedGCN2:
+    """2-layer GCN inference  out = A*(relu(A*(X*W1))*W2)  on G GPUs (NEXT-3): two
+    ShardedGCNLayer, the hidden rows never leave their rank; between the layers one
+    library kernel applies the ReLU and converts to bf16 (mps_relu_to_bf16).  X_rows:
+    this rank's rows [X_g, X_{g+1}) of X (bf16); W1: F x H, W2: H x C (torch, any dtype).
+    Returns this rank's output rows (fp32)."""
+
+    def __init__(self, row_ptr, col_idx, val, n, W1, W2, rank, world, device, tile_cols=64,
+                 group=None, peers1=None, peers2=None, **kw):
+        F, H = W1.shape
+        C = W2.shape[1]
+        self.W1t = W1.t().contiguous().to(device=device, dtype=torch.bfloat16)
+        self.W2t = W2.t().contiguous().to(device=device, dtype=torch.bfloat16)
+        self.l1 = ShardedGCNLayer(row_ptr, col_idx, val, n, F, H, rank, world, device,
+                                  tile_cols=tile_cols, group=group, peers=peers1, **kw)
+        self.l2 = ShardedGCNLayer(row_ptr, col_idx, val, n, H, C, rank, world, device,
+                                  tile_cols=tile_cols, group=group, peers=peers2, **kw)
+        rows = max(self.l1.r1 - self.l1.r0, 1)
+        self.Hb = torch.empty((rows, H), dtype=torch.bfloat16, device=device)
+
+    def hidden(self, stream=None):
+        """relu(layer-1 rows) -> bf16, the next combination's input (one library kernel)."""
+        rows = self.l1.r1 - self.l1.r0
+        C1 = self.l1.sh.C
+        L.mps_relu_to_bf16(_p(C1) if rows else None, rows, C1.shape[1], C1.stride(0),
+                           _p(self.Hb) if rows else None, self.Hb.stride(0), _stream(stream))
+        return self.Hb[:rows]
+
+    def __call__(self, X_rows, s_xw=None, s_agg=None):
+        s_agg = s_agg or torch.cuda.current_stream()
+        self.l1(X_rows, self.W1t, s_xw=s_xw, s_agg=s_agg)
+        H = self.hidden(s_agg)
+        return self.l2(H, self.W2t, s_xw=s_xw, s_agg=s_agg)
+
+    def close(self):
+        self.l1.close()
+        self.l2.close()

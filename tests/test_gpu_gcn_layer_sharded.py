@@ -112,3 +112,63 @@ def test_sharded_gcn_layer_two_processes_ipc(tmp_path):
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     oks = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(oks) == 2 and all('"ok": true' in l for l in oks), r.stdout
+
+
+def _bf16_rne(a):
+    """fp32 -> bf16 round-to-nearest-even (the kernels' __float2bfloat16_rn), as float64."""
+    u = np.ascontiguousarray(a, np.float32).view(np.uint32).astype(np.uint64)
+    u = (u + 0x7FFF + ((u >> 16) & 1)) & 0xFFFF0000
+    return u.astype(np.uint32).view(np.float32).astype(np.float64)
+
+
+@pytest.mark.parametrize("world", [1, 2, 3])
+def test_sharded_gcn2_loopback(world):
+    """out = A*(relu(A*(X*W1))*W2) with the bf16 roundings at the same three points as the
+    kernels (B1, H, B2); integer inputs keep every fp32 sum exact -> bit-exact."""
+    rs = np.random.RandomState(world)
+    n, F, Hd, Cd = 600, 24, 32, 16
+    rl = rs.randint(0, 9, size=n).astype(np.int32)
+    rl[rs.randint(n)] = 400
+    g = G.random_csr(n, n, rl, 11)
+    gen = torch.Generator().manual_seed(world)
+    X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
+    W1 = torch.randint(-1, 2, (F, Hd), generator=gen).to(torch.bfloat16)
+    W2 = torch.randint(-1, 2, (Hd, Cd), generator=gen).to(torch.bfloat16)
+    B1 = _bf16_rne(X.double().numpy() @ W1.double().numpy())
+    C1 = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B1, want_bound=False)
+    Hh = _bf16_rne(np.maximum(C1, 0.0))
+    B2 = _bf16_rne(Hh @ W2.double().numpy())
+    ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B2, want_bound=False)
+
+    def peers(N):
+        Bs = [torch.empty((n, N), dtype=torch.bfloat16, device="cuda") for _ in range(world)]
+        sg = [torch.zeros(int(M.mps_signal_bytes()), dtype=torch.uint8, device="cuda")
+              for _ in range(world)]
+        bx = [torch.zeros(int(M.mps_shard_mailbox_bytes(N)), dtype=torch.uint8, device="cuda")
+              for _ in range(world)]
+        keep.extend(Bs + sg + bx)
+        return [dict(replicas=[b.data_ptr() for b in Bs], signals=[t.data_ptr() for t in sg],
+                     mailboxes=[t.data_ptr() for t in bx], B=Bs[r]) for r in range(world)]
+    keep = []
+    p1, p2 = peers(Hd), peers(Cd)
+    nets = [M.ShardedGCN2(g.row_ptr, g.col_idx, g.val, n, W1.cuda(), W2.cuda(), r, world,
+                          "cuda", tile_cols=16, peers1=p1[r], peers2=p2[r], items_per_part=19,
+                          min_parts=1) for r in range(world)]
+    Xd = X.cuda()
+    s_xw, s_agg = torch.cuda.Stream(), torch.cuda.Stream()
+    for step in range(2):
+        for net in nets:                                  # layer 1, loopback order
+            net.l1.replicate(Xd[net.l1.r0:net.l1.r1], net.W1t, s_xw)
+        for slot in range(len(nets[0].l1.tiles)):
+            for net in nets:
+                net.l1.aggregate_tile(slot, s_agg)
+        Hs = [net.hidden(s_agg) for net in nets]
+        s_xw.wait_stream(s_agg)
+        for net, Hr in zip(nets, Hs):                     # layer 2
+            net.l2.replicate(Hr, net.W2t, s_xw)
+        for slot in range(len(nets[0].l2.tiles)):
+            for net in nets:
+                net.l2.aggregate_tile(slot, s_agg)
+        torch.cuda.synchronize()
+        out = np.concatenate([net.l2.sh.C[: net.l2.sh.rows].cpu().numpy() for net in nets])
+        assert np.array_equal(out.astype(np.float64), ref), step
