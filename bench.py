@@ -553,11 +553,20 @@ def main():
         seg_bytes = alg_bytes(sh.rows, y1 - y0, K, b_elt)
     seg_gbs = seg_bytes / (t_seg * 1e-3) / 1e9
     traffic = None
+    units = None
     prof = os.path.join(ROOT, "profiles", "traffic.json")
     key = "%s-k%d-%s-%s" % (name, K, args.dtype, args.fixup)
     if os.path.exists(prof) and world == 1:
         with open(prof) as f:
-            traffic = json.load(f).get(key)
+            tj = json.load(f)
+            traffic = tj.get(key)
+            u = tj.get("_units", {}).get(key)
+            if u:   # ncu of the same kernel: which unit binds (B in L2 -> L2, else DRAM)
+                units = dict(u, source="ncu --set full, profiles/r01 (traffic.json)",
+                             note=("B fits in L2: the algorithmic-byte fraction exceeds 1; "
+                                   "the binding unit is L2 (lts_throughput_pct)")
+                             if b_elt * g.n * K <= 0.5 * l2 else
+                             "B exceeds L2: DRAM-bound gathers (dram traffic above)")
 
     # cuSPARSE on the same A, B (reference point; not the product)
     cus = None
@@ -706,7 +715,7 @@ def main():
                          "achieved": seg_gbs, "peak": hbm_peak, "unit": "GB/s",
                          "frac": seg_gbs / hbm_peak, "traffic": traffic,
                          "algorithmic_bytes_per_launch": int(seg_bytes),
-                         "peak_source": peak_src},
+                         "peak_source": peak_src, "units": units},
             "b_replication": ({"ms": b_rep_ms, "bytes_per_rank_received": int(
                 (world - 1) * (-(-g.n // world)) * K * b_elt), "collective": "all_gather_into_tensor",
                 "in_step": False, "fused_xw": xw_rep,
