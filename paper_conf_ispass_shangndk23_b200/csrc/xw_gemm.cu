@@ -535,13 +535,16 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
             stages = stages > max_stages ? max_stages : stages;
             stages = stages < 2 ? 2 : stages;
             const size_t smem = fixed + wb(nh) + (size_t)stages * a_bytes;
-            static bool pattr = false;
-            if (!pattr) {
+            // function attributes are per device: set once for each
+            static bool pattr[64] = {false};
+            int dev = 0;
+            if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) dev = 0;
+            if (!pattr[dev]) {
                 cudaError_t e = cudaFuncSetAttribute(xw_persistent_kernel,
                                                      cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                      (int)budget);
                 if (e != cudaSuccess) return e;
-                pattr = true;
+                pattr[dev] = true;
             }
             CUtensorMap mws;
             if (nh != N && !make_map(&mws, Wt, N, F, ldw, nh)) return cudaErrorNotSupported;
@@ -566,13 +569,15 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
     stages = stages < 2 ? 2 : (stages > kXwMaxStages ? kXwMaxStages : stages);
     if (stages > nk) stages = nk < 2 ? 2 : nk;
     const size_t smem = 1024 + (size_t)stages * stage_bytes + 256;
-    static bool attr = false;
-    if (!attr) {
+    static bool attr[64] = {false};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) dev = 0;
+    if (!attr[dev]) {
         cudaError_t e = cudaFuncSetAttribute(
             xw_gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
             (int)(1024 + kXwMaxStages * (kXwBM * kXwBK * 2 + 256 * kXwBK * 2) + 256));
         if (e != cudaSuccess) return e;
-        attr = true;
+        attr[dev] = true;
     }
     const unsigned grid = (unsigned)((n + kXwBM - 1) / kXwBM);
     xw_gemm_kernel<<<grid, kXwThreads, smem, s>>>(mx, mw, n, (int)F, N, stages, dst, ldb);
