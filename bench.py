@@ -30,6 +30,18 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "SpMM GFLOP/s (2·nnz·K) & HBM GB/s vs 8 TB/s at 1/2/4/8 B200"
+# The paper's own results: ratios on other hardware, context only
+PAPER_CONTEXT = {
+    "hardware": "NVIDIA Quadro RTX 6000 (Turing sm_75, 72 SMs, 672 GB/s), fp32 presumed (P:159)",
+    "speedups": {
+        "vs GNNAdvisor, geomean over 22 Table-II graphs, K=16": "1.85x (P:230)",
+        "vs GNNAdvisor-opt": "+31% (P:230)",
+        "online scheduling overhead, 2-layer GCN, geomean": "~2% (P:282)",
+        "online overhead Cora / com-Amazon": "10% / <1% (P:282)",
+    },
+    "absolute_numbers": None,
+    "note": "the paper prints no absolute time or GFLOP/s; not a target (vs_baseline null)",
+}
 FALLBACK_HBM_GBS = 6650.0   # B200_PROFILING.md fallback, used only without MEASURED_PEAKS.json
 
 
@@ -54,6 +66,8 @@ def parse():
                          "several ranks on one GPU)")
     ap.add_argument("--no-cusparse", action="store_true",
                     help="skip the cuSPARSE reference point (N=1, fp32)")
+    ap.add_argument("--no-l2-probe", action="store_true",
+                    help="skip the live L2 read-bandwidth ceiling (roofline.units)")
     ap.add_argument("--tails", default="auto", choices=["auto", "p2p", "nccl"],
                     help="N>1 tail exchange: p2p = fused into the final kernel over peer "
                          "memory (auto: p2p if it sets up and cross-checks, else nccl)")
@@ -568,6 +582,31 @@ def main():
                              if b_elt * g.n * K <= 0.5 * l2 else
                              "B exceeds L2: DRAM-bound gathers (dram traffic above)")
 
+    # live L2 probes (tools/l2_probe.cu): where B fits in L2 the gathers are bound by
+    # L2 -> SM bandwidth; a bare random-gather loop and a streaming read of an L2-resident
+    # table show what plain code reaches on this box, beside the kernel's own rate
+    if world == 1 and not args.no_l2_probe:
+        try:
+            import __graft_entry__
+            lp = ctypes.CDLL(__graft_entry__.build_l2_probe())
+            res = {}
+            for mode, key in ((0, "gather_256B"), (1, "stream")):
+                gb, pm = ctypes.c_float(), ctypes.c_float()
+                rc = lp.l2_probe_read_gbs2(ctypes.c_int64(48 << 20), ctypes.c_int32(256),
+                                           ctypes.c_int32(mode), ctypes.byref(gb),
+                                           ctypes.byref(pm))
+                if rc == 0:
+                    res[key] = round(gb.value, 1)
+            torch.cuda.synchronize(dev)
+            if res:
+                units = dict(units or {})
+                units["l2_probe_gbs"] = res
+                units["l2_probe_source"] = ("measured live: tools/l2_probe.cu, 48 MB L2-resident "
+                                            "table, 16-B no-L1 loads, best of 3 grid shapes")
+                units["segment_vs_l2_probe"] = seg_gbs / max(res.values())
+        except Exception as e:  # pragma: no cover
+            units = dict(units or {}, l2_probe_error=str(e)[:200])
+
     # cuSPARSE on the same A, B (reference point; not the product)
     cus = None
     if world == 1 and args.dtype == "f32" and not args.no_cusparse:
@@ -724,6 +763,7 @@ def main():
             "e2e": e2e,
             "e2e_graph_resident": e2e_res,
             "cusparse": cus,
+            "paper_context": PAPER_CONTEXT,
             "gpu_launches": int(launches_per_step * args.steps),
             "clocks": clk,
         }

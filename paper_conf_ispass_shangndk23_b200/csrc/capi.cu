@@ -788,6 +788,151 @@ mps_status mps_spmm_host_workspace_bytes(const mps_csr *A_host, int32_t K, int32
     return MPS_OK;
 }
 
+// Pipelined end-to-end call (atomic fix-up): the H2D of A is cut into NC chunks at
+// merge-path segment boundaries p_c, so the segment kernel of chunk c overlaps the copy
+// of chunk c+1, and the rows chunk c finalises go back D2H while later chunks still
+// copy in (PCIe is full duplex).  Chunk c covers diagonals [p_c L, p_{c+1} L); the host
+// finds their coordinates (x_c, y_c) with the same search as the shard bounds, so the
+// chunk's non-zeros are exactly [y_c, y_{c+1}) = [cy[p_c], cy[p_{c+1}]) of the device
+// partition (Alg. 1 and its closed form, reading R2).  Rows [x_c, x_{c+1}) are final
+// after chunks 0..c: a row's end item lies on a diagonal below d_{c+1}, and a row cut
+// at x_{c+1} belongs to the next range.  One partition (+ cut-row zeroing) launch over
+// all P segments serves every chunk, so the result is the one mps_spmm_online gives.
+namespace {
+struct AuxStreams {
+    cudaStream_t comp = nullptr, d2h = nullptr;
+};
+AuxStreams aux_streams() {
+    static AuxStreams cache[64];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return AuxStreams{};
+    if (!cache[dev].comp) {
+        cudaStream_t a = nullptr, b = nullptr;
+        if (cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking) != cudaSuccess) return AuxStreams{};
+        if (cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking) != cudaSuccess) {
+            cudaStreamDestroy(a);
+            return AuxStreams{};
+        }
+        cache[dev].d2h = b;
+        cache[dev].comp = a;
+    }
+    return cache[dev];
+}
+
+bool getenv_flag(const char *name) {
+    const char *e = getenv(name);
+    return e && atoi(e) != 0;
+}
+
+int64_t host_chunk_bytes() {
+    const char *e = getenv("MPS_HOST_CHUNK_BYTES");   // read per call (tests vary it)
+    const long long x = e ? atoll(e) : 0;
+    return (int64_t)(x > 0 ? x : (32ll << 20));
+}
+}  // namespace
+
+static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int32_t b_dtype,
+                                 int64_t ldb, int32_t K, float *C_host, int64_t ldc,
+                                 int64_t P, int64_t L, const Vec &v, const HostLayout &h,
+                                 char *w, cudaStream_t s) {
+    const AuxStreams ax = aux_streams();
+    if (!ax.comp) return fail(MPS_ERR_CUDA, "auxiliary streams");
+    const int64_t m = A_host->m, nnz = A_host->nnz, M = m + nnz;
+    int64_t nc = (nnz * 8 + host_chunk_bytes() - 1) / host_chunk_bytes();
+    if (nc < 1) nc = 1;
+    if (nc > 64) nc = 64;
+    if (nc > P) nc = P;
+    std::vector<int64_t> pc(nc + 1), xc(nc + 1), yc(nc + 1);
+    for (int64_t c = 0; c <= nc; ++c) {
+        pc[c] = (P * c) / nc;
+        const int64_t d = pc[c] * L < M ? pc[c] * L : M;
+        xc[c] = host_diag_x(A_host->row_ptr, m, nnz, d);
+        yc[c] = d - xc[c];
+    }
+    const size_t bbytes = (size_t)A_host->n * (size_t)ldb * elt_bytes(b_dtype);
+    int32_t *rp = (int32_t *)(w + h.rp);
+    int32_t *ci = (int32_t *)(w + h.ci);
+    float *va = (float *)(w + h.val);
+    float *C = (float *)(w + h.C);
+    const size_t xb = align_up((size_t)(P + 1) * 4, 256);
+    int32_t *cx = (int32_t *)(w + h.ws);
+    int32_t *cy = (int32_t *)(w + h.ws + xb);
+
+    std::vector<cudaEvent_t> ev(2 * nc + 3, nullptr);
+    for (auto &e : ev)
+        if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) {
+            for (auto &f : ev) if (f) cudaEventDestroy(f);
+            return fail(MPS_ERR_CUDA, "event create");
+        }
+    cudaEvent_t ev_rp = ev[0], ev_B = ev[1], ev_end = ev[2];
+    cudaEvent_t *ev_A = &ev[3], *ev_done = &ev[3 + nc];
+    mps_status st = MPS_OK;
+    auto chk = [&](cudaError_t e, const char *where) {
+        if (e != cudaSuccess && st == MPS_OK) st = cuda_fail(e, where);
+        return st == MPS_OK;
+    };
+    // copy stream (the caller's): row_ptr, B, then A chunk by chunk
+    chk(cudaMemcpyAsync(rp, A_host->row_ptr, (size_t)(m + 1) * 4, cudaMemcpyHostToDevice, s),
+        "H2D row_ptr");
+    chk(cudaEventRecord(ev_rp, s), "event");
+    if (bbytes) chk(cudaMemcpyAsync(w + h.B, B_host, bbytes, cudaMemcpyHostToDevice, s), "H2D B");
+    chk(cudaEventRecord(ev_B, s), "event");
+    for (int64_t c = 0; c < nc && st == MPS_OK; ++c) {
+        const size_t n = (size_t)(yc[c + 1] - yc[c]) * 4;
+        if (n) {
+            chk(cudaMemcpyAsync(ci + yc[c], A_host->col_idx + yc[c], n, cudaMemcpyHostToDevice, s),
+                "H2D col_idx");
+            chk(cudaMemcpyAsync(va + yc[c], A_host->val + yc[c], n, cudaMemcpyHostToDevice, s),
+                "H2D val");
+        }
+        chk(cudaEventRecord(ev_A[c], s), "event");
+    }
+    // compute stream: one partition (+ cut-row zeroing), then the segments chunk by chunk
+    chk(cudaStreamWaitEvent(ax.comp, ev_rp, 0), "wait");
+    if (st == MPS_OK)
+        chk(mps::launch_partition<int32_t>(rp, m, nnz, 0, M, P, L, cx, cy, C, ldc, 0, K, -1,
+                                           nullptr, ax.comp), "partition kernel");
+    chk(cudaStreamWaitEvent(ax.comp, ev_B, 0), "wait");
+    for (int64_t c = 0; c < nc && st == MPS_OK; ++c) {
+        chk(cudaStreamWaitEvent(ax.comp, ev_A[c], 0), "wait");
+        if (pc[c + 1] > pc[c]) {
+            mps::SegArgsT<int32_t> a{};
+            a.rp = rp;
+            a.col = ci;
+            a.val = va;
+            a.B = w + h.B;
+            a.ldb = ldb;
+            a.C = C;
+            a.ldc = ldc;
+            a.row_base = 0;
+            a.m = (int32_t)m;
+            a.cx = cx + pc[c];
+            a.cy = cy + pc[c];
+            a.P = pc[c + 1] - pc[c];
+            a.tail_row = -1;
+            a.tail = nullptr;
+            a.nnz_end = nnz;
+            a.hot = nullptr;
+            a.relu = 0;
+            st = run_segments(a, b_dtype, K, v, mps::FIX_ATOMIC, nullptr, ax.comp);
+        }
+        chk(cudaEventRecord(ev_done[c], ax.comp), "event");
+    }
+    // D2H stream: rows [x_c, x_{c+1}) once chunk c is done (the last chunk: up to m)
+    for (int64_t c = 0; c < nc && st == MPS_OK; ++c) {
+        const int64_t r0 = xc[c], r1 = (c + 1 == nc) ? m : xc[c + 1];
+        chk(cudaStreamWaitEvent(ax.d2h, ev_done[c], 0), "wait");
+        if (r1 > r0)
+            chk(cudaMemcpyAsync(C_host + r0 * ldc, C + r0 * ldc, (size_t)(r1 - r0) * ldc * 4,
+                                cudaMemcpyDeviceToHost, ax.d2h), "D2H C");
+    }
+    // join: the caller's stream sees the whole call
+    chk(cudaEventRecord(ev_end, ax.d2h), "event");
+    chk(cudaStreamWaitEvent(s, ev_end, 0), "wait");
+    for (auto &e : ev) cudaEventDestroy(e);   // released once the recorded work completes
+    return st;
+}
+
 mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dtype,
                          int64_t ldb, int32_t K, float *C_host, int64_t ldc,
                          int64_t items_per_part, int64_t min_parts, int32_t fixup,
@@ -805,6 +950,15 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, h.total);
     cudaStream_t s = (cudaStream_t)stream;
     char *w = (char *)device_workspace;
+    if (resolve_fix(fixup) == mps::FIX_ATOMIC && hot_budget_rows(A_host->n, K, b_dtype) < 0 &&
+        !getenv_flag("MPS_HOST_SERIAL")) {
+        int64_t P, L;
+        if ((st = plan_impl(A_host->m, A_host->nnz, K, b_dtype, items_per_part, min_parts, &P,
+                            &L, false)))
+            return st;
+        const Vec v = choose_vec(K, b_dtype, w + h.B, ldb, (float *)(w + h.C), ldc, A_host->n);
+        return host_pipelined(A_host, B_host, b_dtype, ldb, K, C_host, ldc, P, L, v, h, w, s);
+    }
     const size_t bbytes = (size_t)A_host->n * (size_t)ldb * elt_bytes(b_dtype);
     MPS_CUDA(cudaMemcpyAsync(w + h.rp, A_host->row_ptr, (size_t)(A_host->m + 1) * 4,
                              cudaMemcpyHostToDevice, s), "H2D row_ptr");

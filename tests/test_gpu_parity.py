@@ -443,6 +443,42 @@ def test_spmm_host_end_to_end():
     assert O.check(C.numpy(), ref, bnd)["ok"]
 
 
+@pytest.mark.parametrize("chunk", [1, 4096, 65536, 0])
+@pytest.mark.parametrize("case", ["pubmed", "evil", "empty_rows", "no_nnz"])
+def test_spmm_host_pipelined_chunks(monkeypatch, chunk, case):
+    """mps_spmm_host in atomic mode pipelines the H2D of A in merge-path chunks with the
+    segment kernels and the D2H of finished rows (MPS_HOST_CHUNK_BYTES sets the chunk
+    size; 1 byte = the 64-chunk cap).  Integer inputs: bit-exact against the oracle and
+    against the serial path (MPS_HOST_SERIAL=1), for rows cut by every chunk boundary."""
+    rs = np.random.RandomState(7)
+    if case == "pubmed":
+        g = G.workload("pubmed")
+        g = G.random_csr(g.m, g.n, np.diff(g.row_ptr).astype(np.int32), 11)
+    elif case == "evil":          # one row spanning many chunks, short rows around it
+        rl = rs.randint(0, 6, size=3000).astype(np.int32)
+        rl[1500] = 40000
+        g = G.random_csr(3000, 60000, rl, 12)
+    elif case == "empty_rows":
+        rl = np.where(rs.rand(5000) < 0.8, 0, rs.randint(1, 30, size=5000)).astype(np.int32)
+        g = G.random_csr(5000, 700, rl, 13)
+    else:
+        g = G.random_csr(300, 50, np.zeros(300, np.int32), 14)
+    pin = lambda a: torch.from_numpy(a).pin_memory()
+    for K, dt in ((64, torch.float32), (16, torch.float32), (32, torch.bfloat16)):
+        B = G.dense_int(g.n, K, seed=K + 1)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        Bh = torch.from_numpy(B).to(dt).pin_memory()
+        monkeypatch.setenv("MPS_HOST_CHUNK_BYTES", str(chunk))
+        for cost in (0, 24):
+            C = M.spmm_host(pin(g.row_ptr), pin(g.col_idx), pin(g.val), g.n, Bh,
+                            items_per_part=cost, min_parts=1 if cost else 0)
+            assert np.array_equal(C.numpy().astype(np.float64), ref), (K, dt, cost)
+        monkeypatch.setenv("MPS_HOST_SERIAL", "1")
+        Cs = M.spmm_host(pin(g.row_ptr), pin(g.col_idx), pin(g.val), g.n, Bh)
+        monkeypatch.delenv("MPS_HOST_SERIAL")
+        assert np.array_equal(Cs.numpy(), C.numpy())
+
+
 @pytest.mark.parametrize("fixup", ["atomic", "carry"])
 def test_spmm_host_dense_graph_resident(fixup):
     g = G.workload("pubmed")

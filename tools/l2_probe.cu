@@ -1,0 +1,117 @@
+// l2_probe.cu -- live L2 -> SM read ceiling for the bench's roofline (SURVEY.md
+// sec. 8(d): "L2->SM gather throughput" bounds the path where B fits in L2, e.g. Reddit
+// K=64).  A table of `bytes` (< L2) is made resident, then every warp gathers rows of
+// `row_bytes` at random (a hash of warp and iteration, 16 B per lane, L1 no_allocate,
+// U gathers in flight per lane) -- the a3 access pattern without the SpMM's
+// bookkeeping.  mode 1 streams the table instead (grid-stride, coalesced).  Reports the
+// best read GB/s over a few grid shapes.  NOT part of the product: libmpspmm never
+// links it; bench.py loads it only for roofline.units.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+__device__ __forceinline__ uint32_t mix32(uint32_t x) {
+    x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
+    return x;
+}
+
+__device__ __forceinline__ uint4 ldg_na(const uint4 *p) {
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+
+template <int U>
+__global__ void __launch_bounds__(256) l2_gather(const uint4 *__restrict__ tab, uint32_t nrows,
+                                                 uint32_t row16, int iters, uint32_t *sink) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t rows_per_instr = 32 / row16;            // row16 = 16-B words per row
+    const uint32_t grp = lane / row16, lr = lane % row16;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    uint32_t acc = 0;
+    uint32_t h = mix32(warp * 0x9E3779B9u + 1);
+    for (int it = 0; it < iters; ++it) {
+        uint4 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint32_t r = mix32(h + (uint32_t)(u * rows_per_instr + grp)) % nrows;
+            v[u] = ldg_na(tab + (uint64_t)r * row16 + lr);
+        }
+        h = mix32(h + (uint32_t)it);
+#pragma unroll
+        for (int u = 0; u < U; ++u) acc ^= v[u].x ^ v[u].y ^ v[u].z ^ v[u].w;
+    }
+    if (acc == 0x9e3779b9u) sink[0] = acc;
+}
+
+__global__ void __launch_bounds__(256) l2_stream(const uint4 *__restrict__ buf, int64_t n16,
+                                                 int passes, uint32_t *sink) {
+    uint32_t acc = 0;
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int p = 0; p < passes; ++p)
+        for (int64_t i = tid; i < n16; i += stride) {
+            const uint4 v = ldg_na(buf + i);
+            acc ^= v.x ^ v.y ^ v.z ^ v.w;
+        }
+    if (acc == 0x9e3779b9u) sink[0] = acc;
+}
+
+// mode 0: random row gathers (row_bytes in {16..512}); mode 1: streaming read.
+// Returns 0 on success; *gbs = best bytes read / time over the tried grid shapes.
+extern "C" int l2_probe_read_gbs2(int64_t bytes, int32_t row_bytes, int32_t mode, float *gbs,
+                                  float *ms) {
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (row_bytes < 16 || row_bytes > 512 || (row_bytes & (row_bytes - 1))) return 3;
+    const int64_t n16 = bytes / 16;
+    const uint32_t row16 = (uint32_t)row_bytes / 16;
+    const uint32_t nrows = (uint32_t)(n16 / row16);
+    uint4 *buf = nullptr;
+    uint32_t *sink = nullptr;
+    if (cudaMalloc(&buf, n16 * 16) != cudaSuccess) return 1;
+    if (cudaMalloc(&sink, 4) != cudaSuccess) { cudaFree(buf); return 1; }
+    cudaMemset(buf, 1, n16 * 16);
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    float best = 0.f, best_ms = 0.f;
+    const int per_sm[3] = {3, 4, 8};
+    for (int c = 0; c < 3; ++c) {
+        const int grid = sms * per_sm[c];
+        const int iters = 400;
+        const int passes = 20;
+        if (mode == 0) l2_gather<8><<<grid, 256>>>(buf, nrows, row16, 20, sink);
+        else l2_stream<<<grid, 256>>>(buf, n16, 1, sink);       // make it resident
+        for (int rep = 0; rep < 3; ++rep) {
+            cudaEventRecord(e0);
+            double moved;
+            if (mode == 0) {
+                l2_gather<8><<<grid, 256>>>(buf, nrows, row16, iters, sink);
+                moved = (double)grid * 256 * 16 * 8 * iters;   // 16 B per lane per gather
+            } else {
+                l2_stream<<<grid, 256>>>(buf, n16, passes, sink);
+                moved = (double)n16 * 16 * passes;
+            }
+            cudaEventRecord(e1);
+            cudaEventSynchronize(e1);
+            float t = 0.f;
+            cudaEventElapsedTime(&t, e0, e1);
+            const float g = (float)(moved / (t * 1e-3) / 1e9);
+            if (g > best) { best = g; best_ms = t; }
+        }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(buf);
+    cudaFree(sink);
+    *gbs = best;
+    *ms = best_ms;
+    return cudaGetLastError() == cudaSuccess ? 0 : 2;
+}
+
+extern "C" int l2_probe_read_gbs(int64_t bytes, int passes, float *gbs, float *ms) {
+    (void)passes;
+    return l2_probe_read_gbs2(bytes, 256, 0, gbs, ms);
+}
