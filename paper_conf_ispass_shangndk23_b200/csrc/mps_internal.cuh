@@ -75,6 +75,7 @@ struct SegArgsT {
     int32_t relu;        // epilogue: 1 = C = max(C, 0) (complete rows at the store; cut rows
                          // by launch_relu_split after the atomics, or in the carry reduce)
     TailMail mail;       // a6 peer-memory tail exchange (mail.on == 0: none)
+    unsigned *claim;     // set by the launcher: dynamic segment claims {next, done} or NULL
 };
 using SegArgs = SegArgsT<int32_t>;
 using SegArgs64 = SegArgsT<int64_t>;

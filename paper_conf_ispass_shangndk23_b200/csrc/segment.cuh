@@ -1,4 +1,5 @@
 #pragma once
+#include <atomic>
 #include <cstdlib>
 // segment.cuh -- a3 (+ a4 partial rows): the merge-path segment kernel template (Alg. 2,
 // PAPER.md P:100-131, sec. III-B/C P:121-147).  Instantiated per (B dtype, fix-up) in
@@ -100,8 +101,10 @@ segment_kernel(const SegArgsT<IT> a) {
 
     const uint64_t pol_last = a.l2_hints ? policy_evict_last() : policy_evict_normal();
     const uint64_t pol_first = a.l2_hints ? policy_evict_first() : policy_evict_normal();
-    const int64_t wid = (int64_t)blockIdx.x * kWarps + warp;
-    const int64_t wstride = (int64_t)gridDim.x * kWarps;
+    // segment indices are 32-bit (the launcher rejects P >= 2^31 - 2^20)
+    const int wid = (int)blockIdx.x * kWarps + warp;
+    const int wstride = (int)gridDim.x * kWarps;
+    const int nseg = (int)a.P;
 
     const IT *__restrict__ rp = a.rp;
     const int32_t *__restrict__ col = a.col;
@@ -132,13 +135,27 @@ segment_kernel(const SegArgsT<IT> a) {
     // TMA may not read past the last 16-B boundary inside [.., nnz_end)
     const int64_t lim4 = a.nnz_end - (int64_t)(((uintptr_t)(col + a.nnz_end) & 15u) >> 2);
 
-    // ---------------- producer: one chunk ahead, across this warp's segments ----------
-    int64_t pseg = wid;
+    // ---------------- this warp's sequence of segments ---------------------------------
+    // static: wid, wid + wstride, ...; dynamic (a.claim != nullptr): each warp claims its
+    // next segment from a grid-wide counter when it starts the current one, so warps
+    // that drew cheap segments take more (load balance across SMs and dies).  Claims
+    // are issued in increasing order; cur >= P ends the warp's work.
+    auto claim_after = [&](int last) -> int {
+        if (a.claim == nullptr) return last + wstride;
+        unsigned v = 0;
+        if (lane == 0) v = atomicAdd(a.claim, 1u);
+        return (int)__shfl_sync(0xffffffffu, v, 0);
+    };
+    int cur = a.claim == nullptr ? wid : claim_after(0);
+    int nxt = cur < nseg ? claim_after(cur) : nseg;
+
+    // ---------------- producer: one chunk ahead, at most one segment ahead -------------
+    int pseg = cur;
     IT psb = 0;                          // chunk origin of the producer's segment
     int pys = 0, pye = 0;                // its non-zero range, relative to psb
     int pk = 0, pnch = 0, pbuf = 0;
     auto prod_load_seg = [&]() {
-        if (pseg < a.P) {
+        if (pseg < nseg) {
             const IT ys_ = __ldg(a.cy + pseg), ye_ = __ldg(a.cy + pseg + 1);
             psb = seg_origin(ys_);
             pys = (int)(ys_ - psb);
@@ -148,11 +165,13 @@ segment_kernel(const SegArgsT<IT> a) {
         pk = 0;
     };
     auto produce = [&]() {
-        while (pseg < a.P && pk >= pnch) {
-            pseg += wstride;
+        if (pk >= pnch) {                 // move on to the claimed next segment only
+            if (pseg != cur || nxt >= nseg) return;
+            pseg = nxt;
             prod_load_seg();
+            if (pk >= pnch) return;       // it has no non-zeros: resume when it is cur
         }
-        if (pseg >= a.P) return;
+        if (pseg >= nseg) return;
         const int cbr = pk * kCH;
         const int hir = min(pye, cbr + kCH);
         const IT cb = psb + cbr;
@@ -193,7 +212,15 @@ segment_kernel(const SegArgsT<IT> a) {
     uint32_t phase0 = 0, phase1 = 0;
     int cbuf = 0;
 
-    for (int64_t seg = wid; seg < a.P; seg += wstride) {
+    for (; cur < nseg; cur = nxt, nxt = cur < nseg ? claim_after(cur) : nseg) {
+        const int seg = cur;
+        // claims increase, so the producer is at seg, one segment ahead (it moved past
+        // an empty seg), or behind (it stopped at an earlier empty segment): restart it
+        if (pseg < seg) {
+            pseg = seg;
+            prod_load_seg();
+            produce();
+        }
         const int xs = __ldg(a.cx + seg);
         const IT ys64 = __ldg(a.cy + seg);
         const int xe = __ldg(a.cx + seg + 1);
@@ -276,7 +303,7 @@ segment_kernel(const SegArgsT<IT> a) {
                                                     : a.C + ((int64_t)r - a.row_base) * a.ldc,
                                   true);
                 } else {
-                    write_row(a.rec + (seg * 2) * (int64_t)a.kpad, false);
+                    write_row(a.rec + ((int64_t)seg * 2) * a.kpad, false);
                 }
             } else {
                 // complete row (line 15): plain store, no initialisation of C needed
@@ -425,10 +452,47 @@ segment_kernel(const SegArgsT<IT> a) {
                 write_row((xe == a.tail_row) ? a.tail : a.C + ((int64_t)xe - a.row_base) * a.ldc,
                           true);
             else
-                write_row(a.rec + (seg * 2 + (single ? 0 : 1)) * (int64_t)a.kpad, false);
+                write_row(a.rec + ((int64_t)seg * 2 + (single ? 0 : 1)) * a.kpad, false);
+        }
+    }
+    if (a.claim != nullptr) {             // the last CTA resets the counter for reuse
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            if (atomicAdd(a.claim + 1, 1u) == gridDim.x - 1) {
+                a.claim[0] = 0u;
+                a.claim[1] = 0u;
+                __threadfence();
+            }
         }
     }
     if (a.mail.on) tail_mail_epilogue(a.mail);   // a6 tail exchange (last CTA, last tile)
+}
+
+// Dynamic segment claims: self-resetting counter pairs {next, CTAs done}, zero at module
+// load; every launch takes the next slot (round robin over the whole library), so
+// launches in flight at the same time never share one.  One array per translation unit
+// (no relocatable device code); the slot index is global.
+constexpr int kClaimSlots = 1024;
+static __device__ unsigned g_claim[2 * kClaimSlots];
+inline std::atomic<uint32_t> g_claim_next{0};
+
+static unsigned *claim_slots() {
+    static unsigned *cache[64] = {nullptr};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+    if (!cache[dev]) {
+        void *p = nullptr;
+        if (cudaGetSymbolAddress(&p, g_claim) != cudaSuccess) return nullptr;
+        cache[dev] = (unsigned *)p;
+    }
+    return cache[dev];
+}
+
+// MPS_DYN (read per call): 0 = static segment assignment (warp w: w, w + warps, ...)
+static bool dynamic_claims() {
+    const char *e = getenv("MPS_DYN");
+    return e ? atoi(e) != 0 : true;
 }
 
 template <int W, int V, int NR, typename TB, int FIX, typename IT>
@@ -458,7 +522,15 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     const int64_t cap = (int64_t)blocks_per_sm * num_sms();
     const int64_t grid = need < cap ? need : cap;
     if (grid <= 0) return cudaSuccess;
-    segment_kernel<W, V, NR, TB, FIX, IT><<<(unsigned)grid, kBlock, 0, s>>>(a);
+    if (a.P >= (int64_t)0x7ff00000) return cudaErrorInvalidValue;   // 32-bit segment ids
+    SegArgsT<IT> arg = a;
+    arg.claim = nullptr;
+    if (need > grid && dynamic_claims()) {   // more segments than warps: balance them
+        unsigned *base = claim_slots();
+        if (base == nullptr) return cudaErrorInvalidSymbol;
+        arg.claim = base + 2 * (g_claim_next.fetch_add(1u) % kClaimSlots);
+    }
+    segment_kernel<W, V, NR, TB, FIX, IT><<<(unsigned)grid, kBlock, 0, s>>>(arg);
     return cudaGetLastError();
 }
 

@@ -388,6 +388,42 @@ def test_gcn2_tcgen05_combination():
     assert r["ok"], r
 
 
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_dynamic_segment_claims(monkeypatch, fixup):
+    """More segments than resident warps: warps claim segments from a self-resetting
+    grid counter (MPS_DYN=1, default) instead of the static stride (MPS_DYN=0).  Integer
+    inputs bit-exact against the oracle for both, over repeated launches (the counter must
+    come back to zero), empty-row runs, a CUDA-graph replay and the offline entry point."""
+    rs = np.random.RandomState(17)
+    rl = rs.randint(0, 9, size=30000).astype(np.int32)
+    rl[rs.rand(30000) < 0.3] = 0                   # runs of empty rows -> empty segments
+    rl[12345] = 20000                               # a row cut by many segments
+    g = G.random_csr(30000, 5000, rl, 21)
+    A = dev(g)
+    for K, dt in ((64, torch.float32), (16, torch.float32), (32, torch.bfloat16)):
+        B = G.dense_int(5000, K, seed=K)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for dyn in ("1", "0"):
+            monkeypatch.setenv("MPS_DYN", dyn)
+            for cost in (2, 7):
+                for _ in range(3):
+                    C = M.spmm(A, tB(B, dt), fixup=fixup, items_per_part=cost, min_parts=1)
+                    assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (K, dyn, cost)
+                sch = M.Schedule.build(A, K, dt, items_per_part=cost, min_parts=1)
+                C = M.spmm(A, tB(B, dt), schedule=sch, fixup=fixup)
+                assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (K, dyn, cost)
+    monkeypatch.setenv("MPS_DYN", "1")
+    B = G.dense_int(5000, 64, seed=3)
+    ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+    Bd = tB(B)
+    cap = M.CapturedSpMM(A, Bd, fixup=fixup, items_per_part=3, min_parts=1)
+    for _ in range(4):
+        cap.C.fill_(float("nan"))
+        C = cap()
+        torch.cuda.synchronize()
+        assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
+
+
 def test_carry_is_deterministic():
     g = G.workload("pubmed")
     B = tB(G.features("pubmed", 64))

@@ -31,6 +31,24 @@ def run():
                     if not np.array_equal(C.cpu().numpy().astype(np.float64), ref):
                         print("MISMATCH", K, dt, fixup, cost)
                         bad += 1
+    # dynamic segment claims (more segments than resident warps), repeated launches
+    rl = rs.randint(0, 9, size=12000).astype(np.int32)
+    rl[rs.rand(12000) < 0.3] = 0
+    rl[777] = 5000
+    g = G.random_csr(12000, 2000, rl, 77)
+    A = M.CSR(torch.from_numpy(g.row_ptr).cuda(), torch.from_numpy(g.col_idx).cuda(),
+              torch.from_numpy(g.val).cuda(), g.n)
+    for K, dt in ((64, torch.float32), (32, torch.bfloat16)):
+        B = G.dense_int(2000, K, seed=K)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for fixup in ("atomic", "carry"):
+            for _ in range(2):
+                C = M.spmm(A, torch.from_numpy(B).cuda().to(dt), fixup=fixup, items_per_part=2,
+                           min_parts=1)
+                torch.cuda.synchronize()
+                if not np.array_equal(C.cpu().numpy().astype(np.float64), ref):
+                    print("MISMATCH dynamic claims", K, dt, fixup)
+                    bad += 1
     # shard path (loopback)
     g = G.random_csr(80, 60, np.r_[np.ones(40, np.int32), [700], np.ones(39, np.int32)], 3)
     B = G.dense_int(60, 12, seed=1)
