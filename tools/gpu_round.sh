@@ -13,7 +13,7 @@ tail -1 gpurun_out/bench_$TAG.log | cut -c1-300
 if [ "${NCU:-1}" = "1" ]; then
   timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
      --log-file gpurun_out/launches_$TAG.csv python bench.py $BENCH_ARGS --steps 3 --warmup 3 \
-     --e2e-steps 0 --no-cpu-baseline > gpurun_out/ncu_launch_$TAG.log 2>&1
+     --e2e-steps 0 --no-cpu-baseline --no-cusparse --no-l2-probe > gpurun_out/ncu_launch_$TAG.log 2>&1
   for c in ${PROF_CFGS:-reddit:64 reddit:256 products:128 rmat:64}; do
     tools/prof.sh ${TAG}_${c%%:*}_k${c##*:} ${c%%:*} ${c##*:}
   done
