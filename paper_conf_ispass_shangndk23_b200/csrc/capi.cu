@@ -68,6 +68,7 @@ int64_t default_cost(int64_t m, int64_t nnz, int32_t K, int32_t dt) {
 struct Vec {
     int W = 1;     // elements per lane access
     int tile = 0;  // columns per launch (multiple of 32*W)
+    bool deep = false;  // DRAM-bound gathers: the deep-gather instantiation (see below)
 };
 
 static int64_t l2_bytes() {
@@ -88,7 +89,7 @@ static int64_t l2_bytes() {
 // rows) exceeds half the L2, each pass covers 256-byte slices of the B rows, so the L2
 // holds a larger share of every pass's working set (Reddit K=256 fp32: 8.1 -> 6.5 ms).
 Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C, int64_t ldc,
-               int64_t b_rows = 0) {
+               int64_t b_rows = 0, int64_t m = 0, int64_t nnz = 0) {
     const int eb = elt_bytes(dt);
     const int cand_f32[3] = {4, 2, 1};
     const int cand_bf[4] = {8, 4, 2, 1};
@@ -115,16 +116,26 @@ Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C
         if (cand[i] <= max_w && ok(cand[i])) { v.W = cand[i]; v.tile = 32 * cand[i] * max_v; }
     if (v.tile == 0) { v.W = 1; v.tile = 32 * max_v; }
     // MPS_TILE: tuning override of the column-tile width (0 = rule below, -1 = no tiling)
-    static const int env_tile = [] {
-        const char *e = getenv("MPS_TILE");
-        return e ? atoi(e) : 0;
-    }();
+    const char *et = getenv("MPS_TILE");   // read per call (tests vary it)
+    const int env_tile = et ? atoi(et) : 0;
     int tile = 0;
     if (env_tile > 0) tile = env_tile;
     else if (env_tile == 0 && b_rows > 0 &&
              (double)b_rows * K * eb > 0.5 * (double)l2_bytes())
         tile = 256 / eb;
     if (tile > 0 && tile < v.tile && tile < K) v.tile = (tile / v.W > 0 ? tile / v.W : 1) * v.W;
+    // Deep gathers (2x the 16-B gathers in flight per lane, 2 CTAs/SM at 128 registers)
+    // for fp32 256-B row slices when a pass's B slice exceeds half the L2 and rows are
+    // long enough (>= 32 non-zeros on average) for the larger batches to stay on the
+    // fast path: DRAM-bound gathers want more bytes in flight (products K=128 -2.1%,
+    // Reddit K=256 -1.3%); L2-resident B and short rows (R-MAT) lose with it
+    // (profiles/r01/deep_gathers/).  MPS_DEEP=0/1 overrides.
+    const char *ed = getenv("MPS_DEEP");
+    const int kt = v.tile < K ? v.tile : K;
+    if (ed) v.deep = atoi(ed) != 0;
+    else v.deep = b_rows > 0 && m > 0 && nnz >= 32 * m &&
+                  (double)b_rows * kt * eb > 0.5 * (double)l2_bytes();
+    v.deep = v.deep && dt == MPS_DT_F32 && v.W == 4 && kt == 64;
     return v;
 }
 
@@ -225,6 +236,7 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
         a.l2_hints = hints;
         int V, NR;
         tile_geometry(kt, v.W, &V, &NR);
+        a.deep = v.deep && kt == 64 ? 1 : 0;
         mps::SegArgsT<IT> seg_only = a;
         seg_only.mail.on = 0;
         MPS_CUDA(mps::launch_segments(fix == mps::FIX_CARRY ? seg_only : a, dt, v.W, V, NR, fix,
@@ -413,7 +425,7 @@ mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t l
     if (K == 0 || A->m == 0) return MPS_OK;
     if (!coord_x || !coord_y) return fail(MPS_ERR_INVALID, "NULL coordinates");
     const int fix = resolve_fix(fixup);
-    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n, A->m, A->nnz);
     if (fix == mps::FIX_CARRY && workspace_bytes < carry_bytes(num_parts, K, v))
         return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes,
                     carry_bytes(num_parts, K, v));
@@ -546,7 +558,7 @@ mps_status online_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t 
                         sizeof(IT) == 8)))
         return st;
     const int fix = resolve_fix(fixup);
-    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n, A->m, A->nnz);
     const int64_t hot_rows = hot_budget_rows(A->n, K, b_dtype);
     const int64_t nh = hot_rows >= 0 ? A->n : 0;
     const size_t need = online_bytes(P, K, v, fix, nh, sizeof(IT));
@@ -956,7 +968,8 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
         if ((st = plan_impl(A_host->m, A_host->nnz, K, b_dtype, items_per_part, min_parts, &P,
                             &L, false)))
             return st;
-        const Vec v = choose_vec(K, b_dtype, w + h.B, ldb, (float *)(w + h.C), ldc, A_host->n);
+        const Vec v = choose_vec(K, b_dtype, w + h.B, ldb, (float *)(w + h.C), ldc, A_host->n,
+                                 A_host->m, A_host->nnz);
         return host_pipelined(A_host, B_host, b_dtype, ldb, K, C_host, ldc, P, L, v, h, w, s);
     }
     const size_t bbytes = (size_t)A_host->n * (size_t)ldb * elt_bytes(b_dtype);
@@ -1315,7 +1328,8 @@ static mps_status shard_impl(const CSR *A, const void *B, int32_t b_dtype, int64
         if (mail.pull_mask && !C_local) return fail(MPS_ERR_INVALID, "C_local NULL");
     }
     const int fix = resolve_fix(fixup);
-    const Vec v = choose_vec(K, b_dtype, B, ldb, C_local ? C_local : tail_out, ldc, A->n);
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C_local ? C_local : tail_out, ldc, A->n, A->m,
+                             A->nnz);
     if (span == 0) {
         // an empty shard still takes part in the exchange: run the final kernel empty
         if (!mail.on) return MPS_OK;

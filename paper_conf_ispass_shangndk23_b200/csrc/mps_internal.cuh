@@ -76,6 +76,7 @@ struct SegArgsT {
                          // by launch_relu_split after the atomics, or in the carry reduce)
     TailMail mail;       // a6 peer-memory tail exchange (mail.on == 0: none)
     unsigned *claim;     // set by the launcher: dynamic segment claims {next, done} or NULL
+    int32_t deep;        // 1: deep-gather instantiation (fp32, 64-column tile, DRAM-bound B)
 };
 using SegArgs = SegArgsT<int32_t>;
 using SegArgs64 = SegArgsT<int64_t>;

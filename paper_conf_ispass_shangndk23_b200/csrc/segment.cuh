@@ -60,16 +60,17 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
 #endif
-template <int W, int V, typename TB, typename IT>
+template <int W, int V, typename TB, typename IT, bool DEEP = false>
 constexpr int seg_min_blocks() {
+    if constexpr (DEEP) return 2;
     // int64 indices (NEXT-4): fp32 B measured best at 3 CTAs/SM with a few spills
     // (profiles/r01/next4), bf16 B keeps the int32 choice
     return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2
            : (sizeof(TB) == 2 ? MPS_MINB_BF16 : (sizeof(IT) == 8 ? MPS_MINB_I64 : MPS_MINB_F32));
 }
 
-template <int W, int V, int NR, typename TB, int FIX, typename IT>
-__global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB, IT>()))
+template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false>
+__global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB, IT, DEEP>()))
 segment_kernel(const SegArgsT<IT> a) {
     using BV = BVec<TB, W>;
     using raw_t = typename BV::raw;
@@ -79,7 +80,8 @@ segment_kernel(const SegArgsT<IT> a) {
     constexpr int kWords = (W * (int)sizeof(TB) + 3) / 4;
     // per-lane gathers per batch: ~4 KB of B rows in flight per warp
     constexpr int UL00 = (V * kWords >= 8) ? 4 : ((V * kWords >= 4) ? 8 : 16);
-    constexpr int UL0 = (sizeof(TB) == 2 && UL00 / MPS_UL_DIV >= 2) ? UL00 / MPS_UL_DIV : UL00;
+    constexpr int UL0 = (sizeof(TB) == 2 && UL00 / MPS_UL_DIV >= 2) ? UL00 / MPS_UL_DIV
+                                                                    : UL00 * (DEEP ? 2 : 1);
     constexpr int UL = (UL0 * NR > 32) ? (32 / NR > 0 ? 32 / NR : 1) : UL0;
     constexpr int U = UL * NR;                           // non-zeros per batch
     static_assert(kCH % U == 0, "chunk must hold whole batches");
@@ -495,7 +497,7 @@ static bool dynamic_claims() {
     return e ? atoi(e) != 0 : true;
 }
 
-template <int W, int V, int NR, typename TB, int FIX, typename IT>
+template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false>
 static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     static int blocks_per_sm = 0;
     if (blocks_per_sm == 0) {
@@ -508,12 +510,12 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
         }();
         cudaError_t e = cudaSuccess;
         if (carve >= 0) {
-            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT>,
+            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT, DEEP>,
                                      cudaFuncAttributePreferredSharedMemoryCarveout, carve);
             if (e != cudaSuccess) return e;
         }
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX, IT>, kBlock, 0);
+            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX, IT, DEEP>, kBlock, 0);
         if (e != cudaSuccess) return e;
         if (blocks_per_sm < 1) blocks_per_sm = 1;
     }
@@ -530,7 +532,7 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
         if (base == nullptr) return cudaErrorInvalidSymbol;
         arg.claim = base + 2 * (g_claim_next.fetch_add(1u) % kClaimSlots);
     }
-    segment_kernel<W, V, NR, TB, FIX, IT><<<(unsigned)grid, kBlock, 0, s>>>(arg);
+    segment_kernel<W, V, NR, TB, FIX, IT, DEEP><<<(unsigned)grid, kBlock, 0, s>>>(arg);
     return cudaGetLastError();
 }
 
@@ -540,7 +542,10 @@ static cudaError_t dispatch_v(const SegArgsT<IT> &a, int V, int NR, cudaStream_t
     if (V == 1) {
         switch (NR) {
         case 1: return launch_seg<W, 1, 1, TB, FIX, IT>(a, s);
-        case 2: return launch_seg<W, 1, 2, TB, FIX, IT>(a, s);
+        case 2:
+            if constexpr (W == 4 && sizeof(TB) == 4)
+                if (a.deep) return launch_seg<W, 1, 2, TB, FIX, IT, true>(a, s);
+            return launch_seg<W, 1, 2, TB, FIX, IT>(a, s);
         case 4: return launch_seg<W, 1, 4, TB, FIX, IT>(a, s);
         case 8: return launch_seg<W, 1, 8, TB, FIX, IT>(a, s);
         case 16: return launch_seg<W, 1, 16, TB, FIX, IT>(a, s);

@@ -424,6 +424,30 @@ def test_dynamic_segment_claims(monkeypatch, fixup):
         assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
 
 
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_deep_gather_variant(monkeypatch, fixup):
+    """The deep-gather instantiation (2x gathers in flight, 2 CTAs/SM; chosen for fp32
+    256-B row slices when B is DRAM-bound and rows are long) forced on with MPS_DEEP=1:
+    integer inputs bit-exact, untiled K=64 and K=128/192 in 64-column tiles, static and
+    dynamic segment claims."""
+    monkeypatch.setenv("MPS_DEEP", "1")
+    monkeypatch.setenv("MPS_TILE", "64")
+    rs = np.random.RandomState(23)
+    rl = rs.randint(0, 80, size=4000).astype(np.int32)
+    rl[rs.rand(4000) < 0.2] = 0
+    rl[100] = 3000
+    g = G.random_csr(4000, 3500, rl, 31)
+    A = dev(g)
+    for K in (64, 128, 192):
+        B = G.dense_int(3500, K, seed=K)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for dyn in ("1", "0"):
+            monkeypatch.setenv("MPS_DYN", dyn)
+            for cost in (3, 64, 0):
+                C = M.spmm(A, tB(B), fixup=fixup, items_per_part=cost, min_parts=1 if cost else 0)
+                assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (K, dyn, cost)
+
+
 def test_carry_is_deterministic():
     g = G.workload("pubmed")
     B = tB(G.features("pubmed", 64))
