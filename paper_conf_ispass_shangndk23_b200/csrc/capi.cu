@@ -5,6 +5,7 @@
 #include <cstdarg>
 #include <cstdlib>
 #include <type_traits>
+#include <mutex>
 #include <vector>
 
 #include <cuda.h>
@@ -816,8 +817,10 @@ struct AuxStreams {
 };
 AuxStreams aux_streams() {
     static AuxStreams cache[64];
+    static std::mutex mu;
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return AuxStreams{};
+    std::lock_guard<std::mutex> lock(mu);
     if (!cache[dev].comp) {
         cudaStream_t a = nullptr, b = nullptr;
         if (cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking) != cudaSuccess) return AuxStreams{};
