@@ -128,8 +128,8 @@ Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C
     // Deep gathers (2x the 16-B gathers in flight per lane, 2 CTAs/SM at 128 registers)
     // for fp32 256-B row slices when a pass's B slice exceeds half the L2 and rows are
     // long enough (>= 32 non-zeros on average) for the larger batches to stay on the
-    // fast path: DRAM-bound gathers want more bytes in flight (products K=128 -2.1%,
-    // Reddit K=256 -1.3%); L2-resident B and short rows (R-MAT) lose with it
+    // fast path: DRAM-bound gathers want more bytes in flight (products K=128 -3.2%);
+    // L2-resident B (Reddit K=64: +1.7%) and short rows (R-MAT: +10%) lose with it
     // (profiles/r01/deep_gathers/).  MPS_DEEP=0/1 overrides.
     const char *ed = getenv("MPS_DEEP");
     const int kt = v.tile < K ? v.tile : K;
