@@ -69,7 +69,8 @@ constexpr int seg_min_blocks() {
            : (sizeof(TB) == 2 ? MPS_MINB_BF16 : (sizeof(IT) == 8 ? MPS_MINB_I64 : MPS_MINB_F32));
 }
 
-template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false>
+template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false,
+          bool DYN = false>
 __global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB, IT, DEEP>()))
 segment_kernel(const SegArgsT<IT> a) {
     using BV = BVec<TB, W>;
@@ -142,13 +143,17 @@ segment_kernel(const SegArgsT<IT> a) {
     // next segment from a grid-wide counter when it starts the current one, so warps
     // that drew cheap segments take more (load balance across SMs and dies).  Claims
     // are issued in increasing order; cur >= P ends the warp's work.
+    // (a separate instantiation: the claim code alone costs ~4% on small graphs)
     auto claim_after = [&](int last) -> int {
-        if (a.claim == nullptr) return last + wstride;
-        unsigned v = 0;
-        if (lane == 0) v = atomicAdd(a.claim, 1u);
-        return (int)__shfl_sync(0xffffffffu, v, 0);
+        if constexpr (!DYN) {
+            return last + wstride;
+        } else {
+            unsigned v = 0;
+            if (lane == 0) v = atomicAdd(a.claim, 1u);
+            return (int)__shfl_sync(0xffffffffu, v, 0);
+        }
     };
-    int cur = a.claim == nullptr ? wid : claim_after(0);
+    int cur = DYN ? claim_after(0) : wid;
     int nxt = cur < nseg ? claim_after(cur) : nseg;
 
     // ---------------- producer: one chunk ahead, at most one segment ahead -------------
@@ -167,7 +172,12 @@ segment_kernel(const SegArgsT<IT> a) {
         pk = 0;
     };
     auto produce = [&]() {
-        if (pk >= pnch) {                 // move on to the claimed next segment only
+        if constexpr (!DYN) {             // static: skip ahead over empty segments
+            while (pseg < nseg && pk >= pnch) {
+                pseg += wstride;
+                prod_load_seg();
+            }
+        } else if (pk >= pnch) {          // dynamic: move on to the claimed next only
             if (pseg != cur || nxt >= nseg) return;
             pseg = nxt;
             prod_load_seg();
@@ -216,9 +226,9 @@ segment_kernel(const SegArgsT<IT> a) {
 
     for (; cur < nseg; cur = nxt, nxt = cur < nseg ? claim_after(cur) : nseg) {
         const int seg = cur;
-        // claims increase, so the producer is at seg, one segment ahead (it moved past
-        // an empty seg), or behind (it stopped at an earlier empty segment): restart it
-        if (pseg < seg) {
+        // dynamic claims increase, so the producer is at seg, one segment ahead (it moved
+        // past an empty seg), or behind (it stopped at an earlier empty one): restart it
+        if (DYN && pseg < seg) {
             pseg = seg;
             prod_load_seg();
             produce();
@@ -457,7 +467,7 @@ segment_kernel(const SegArgsT<IT> a) {
                 write_row(a.rec + ((int64_t)seg * 2 + (single ? 0 : 1)) * a.kpad, false);
         }
     }
-    if (a.claim != nullptr) {             // the last CTA resets the counter for reuse
+    if constexpr (DYN) {                  // the last CTA resets the counter for reuse
         __syncthreads();
         if (threadIdx.x == 0) {
             __threadfence();
@@ -510,12 +520,15 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
         }();
         cudaError_t e = cudaSuccess;
         if (carve >= 0) {
-            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT, DEEP>,
+            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>,
                                      cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+            if (e == cudaSuccess)
+                e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>,
+                                         cudaFuncAttributePreferredSharedMemoryCarveout, carve);
             if (e != cudaSuccess) return e;
         }
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX, IT, DEEP>, kBlock, 0);
+            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>, kBlock, 0);
         if (e != cudaSuccess) return e;
         if (blocks_per_sm < 1) blocks_per_sm = 1;
     }
@@ -527,12 +540,20 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     if (a.P >= (int64_t)0x7ff00000) return cudaErrorInvalidValue;   // 32-bit segment ids
     SegArgsT<IT> arg = a;
     arg.claim = nullptr;
-    if (need > grid && dynamic_claims()) {   // more segments than warps: balance them
+    bool dyn = false;
+    // dynamic claims pay off from ~4 segments per warp (BASELINE graphs: 10-70 per warp,
+    // 1-6% faster); at 1-3 per warp the opening burst of claims on one counter costs more
+    // than the balance gains (Table-II graphs, profiles/r01/dynamic_claims/)
+    if (a.P >= 4 * grid * warps_per_block && dynamic_claims()) {
         unsigned *base = claim_slots();
         if (base == nullptr) return cudaErrorInvalidSymbol;
         arg.claim = base + 2 * (g_claim_next.fetch_add(1u) % kClaimSlots);
+        dyn = true;
     }
-    segment_kernel<W, V, NR, TB, FIX, IT, DEEP><<<(unsigned)grid, kBlock, 0, s>>>(arg);
+    if (dyn)
+        segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true><<<(unsigned)grid, kBlock, 0, s>>>(arg);
+    else
+        segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false><<<(unsigned)grid, kBlock, 0, s>>>(arg);
     return cudaGetLastError();
 }
 

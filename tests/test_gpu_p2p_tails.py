@@ -10,6 +10,7 @@ two inbox slots and the acknowledgements are exercised).
 """
 import ctypes
 import os
+import re
 import socket
 import subprocess
 import sys
@@ -112,8 +113,9 @@ def test_p2p_tails_two_processes_ipc(tmp_path):
            "--master-addr", "127.0.0.1", "--master-port", str(port), str(w), ROOT]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
-    oks = [l for l in r.stdout.splitlines() if l.startswith("{")]
-    assert len(oks) == 2 and all('"ok": true' in l for l in oks), r.stdout
+    # the two ranks share stdout: their lines may interleave, so match the records
+    oks = re.findall(r'\{"rank": (\d+), "ok": (true|false)\}', r.stdout)
+    assert sorted(int(k) for k, _ in oks) == [0, 1] and all(v == "true" for _, v in oks), r.stdout
 
 
 @pytest.mark.parametrize("tails", ["nccl", "p2p"])

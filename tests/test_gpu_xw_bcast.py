@@ -7,6 +7,7 @@
    real PeerReplicas / xw_replicate path, each process mapping the other's replica.
 """
 import os
+import re
 import socket
 import subprocess
 import sys
@@ -117,5 +118,6 @@ def test_xw_replicate_two_processes_ipc(tmp_path):
            "--master-addr", "127.0.0.1", "--master-port", str(port), str(w), ROOT]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
-    oks = [l for l in r.stdout.splitlines() if l.startswith("{")]
-    assert len(oks) == 2 and all('"ok": true' in l for l in oks), r.stdout
+    # the two ranks share stdout: their lines may interleave, so match the records
+    oks = re.findall(r'\{"rank": (\d+), "ok": (true|false)\}', r.stdout)
+    assert sorted(int(k) for k, _ in oks) == [0, 1] and all(v == "true" for _, v in oks), r.stdout

@@ -19,8 +19,8 @@ import paper_conf_ispass_shangndk23_b200 as M
 from paper_conf_ispass_shangndk23_b200 import _lib as L
 from paper_conf_ispass_shangndk23_b200.api import _p, _stream
 
-KS = (2, 4, 8, 16, 32, 64, 128)
-COSTS = (0, 64, 128, 256, 512, 1024, 2048, 4096)
+KS = tuple(int(x) for x in os.environ.get("SENS_KS", "2 4 8 16 32 64 128").split())
+COSTS = tuple(int(x) for x in os.environ.get("SENS_COSTS", "0 64 128 256 512 1024 2048 4096").split())
 
 
 def replay_ms(fn, reps=20):
