@@ -49,6 +49,21 @@ def run():
                 if not np.array_equal(C.cpu().numpy().astype(np.float64), ref):
                     print("MISMATCH dynamic claims", K, dt, fixup)
                     bad += 1
+    # deep-gather instantiation forced on (fp32, 64-column tiles), static and dynamic
+    os.environ["MPS_DEEP"] = "1"
+    os.environ["MPS_TILE"] = "64"
+    for K in (64, 128):
+        B = G.dense_int(2000, K, seed=K)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for fixup in ("atomic", "carry"):
+            for cost in (2, 0):
+                C = M.spmm(A, torch.from_numpy(B).cuda(), fixup=fixup, items_per_part=cost,
+                           min_parts=1 if cost else 0)
+                torch.cuda.synchronize()
+                if not np.array_equal(C.cpu().numpy().astype(np.float64), ref):
+                    print("MISMATCH deep", K, fixup, cost)
+                    bad += 1
+    del os.environ["MPS_DEEP"], os.environ["MPS_TILE"]
     # shard path (loopback)
     g = G.random_csr(80, 60, np.r_[np.ones(40, np.int32), [700], np.ones(39, np.int32)], 3)
     B = G.dense_int(60, 12, seed=1)
