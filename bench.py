@@ -363,9 +363,15 @@ def main():
     flush = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
     flush_sink = torch.empty(1, dtype=torch.float32, device=dev)
 
+    flush_clean = torch.zeros_like(flush) if args.flush == "write" else None
+
     def do_flush():
         if args.flush == "write":
+            # write 2x L2, then read another 2x L2: the written lines are evicted (and
+            # written back) here, untimed, so the step starts from a cold L2 holding
+            # clean lines instead of paying the flush's write-backs
             flush.zero_()
+            torch.sum(flush_clean, dim=0, out=flush_sink[0])
         elif args.flush == "read":
             torch.sum(flush, dim=0, out=flush_sink[0])
 
@@ -753,7 +759,8 @@ def main():
                 "workload": "%s-k%d" % (name, K), "graph": g.name, "n": g.m, "nnz": g.nnz,
                 "K": K, "b_dtype": args.dtype, "fixup": args.fixup,
                 "num_parts": P, "items_per_part": Lp, "mode": "online (partition every step)",
-                "l2": {"write": "flushed before every timed step (2x L2 write, untimed)",
+                "l2": {"write": "flushed before every timed step (2x L2 write, then 2x L2 read "
+                                 "of a second buffer so no dirty lines remain; untimed)",
                        "read": "flushed before every timed step (2x L2 read, untimed)",
                        "none": "not flushed (col/val > L2)"}[args.flush],
                 "parallelism": "merge-path shards x%d" % world, "graph_sha": g.digest(),

@@ -26,6 +26,8 @@ g = G.workload(wl)
 Bd = torch.from_numpy(G.features(wl, K)).cuda()
 l2 = torch.cuda.get_device_properties(0).L2_cache_size
 flush = torch.empty(2 * l2 // 4, device="cuda")
+flush_clean = torch.zeros_like(flush)
+sink = torch.empty(1, device="cuda")
 res = {"workload": "%s-k%d" % (wl, K), "n": g.m, "nnz": g.nnz, "per_G": {}}
 t1 = None
 ipp = int(os.environ.get("IPP", "0"))
@@ -38,7 +40,8 @@ for world in [int(x) for x in os.environ.get("GS", "1 2 4 8").split()]:
         torch.cuda.synchronize()
         ts = []
         for _ in range(reps):
-            flush.zero_()
+            flush.zero_()                 # bench.py's flush: write 2x L2, read 2x L2
+            torch.sum(flush_clean, dim=0, out=sink[0])
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
             sh.local(Bd)
