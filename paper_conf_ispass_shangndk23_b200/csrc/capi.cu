@@ -112,14 +112,14 @@ Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C
         const int v = e ? atoi(e) : 4;
         return v < 1 ? 1 : (v > 4 ? 4 : v);
     }();
-    // narrow K (fp32): keep >= 4 lanes per B row (NR <= 8 rows per warp instruction).
-    // Fewer rows per instruction mean shorter row-end butterflies and fewer predicated
-    // passes per batch; measured on the 22 Table-II graphs (CUDA-graph replay): K=4
-    // +12%, K=8 +8%, K=2 +4% over 16-B gathers with 16-32 rows per instruction
-    // (profiles/r01/narrow_k/).  MPS_NARROW=0 disables.
+    // narrow K: keep >= 4 lanes per B row (NR <= 8 rows per warp instruction).  Fewer
+    // rows per instruction mean shorter row-end butterflies and fewer predicated passes
+    // per batch; measured on the 22 Table-II graphs (CUDA-graph replay) over 16-B
+    // gathers with 16-32 rows per instruction: fp32 K=2/4/8 +4/12/8%, bf16 K=4/8/16
+    // +11/35/16% (profiles/r01/narrow_k/).  MPS_NARROW=0 disables.
     int wcap = max_w;
     const char *en = getenv("MPS_NARROW");
-    if (dt == MPS_DT_F32 && (!en || atoi(en) != 0)) {
+    if (!en || atoi(en) != 0) {
         int lim = K / 4 < 1 ? 1 : K / 4;
         int p2 = 1;
         while (p2 * 2 <= lim) p2 *= 2;

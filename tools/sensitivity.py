@@ -20,6 +20,7 @@ from paper_conf_ispass_shangndk23_b200 import _lib as L
 from paper_conf_ispass_shangndk23_b200.api import _p, _stream
 
 KS = tuple(int(x) for x in os.environ.get("SENS_KS", "2 4 8 16 32 64 128").split())
+DT = 1 if os.environ.get("SENS_DTYPE", "f32") == "bf16" else 0   # B dtype code
 COSTS = tuple(int(x) for x in os.environ.get("SENS_COSTS", "0 64 128 256 512 1024 2048 4096").split())
 
 
@@ -57,15 +58,17 @@ def main():
         s = _stream()
         for K in KS:
             B = torch.from_numpy(G.features(g.n, K, seed=11)).cuda()
+            if DT:
+                B = B.to(torch.bfloat16)
             C = torch.empty((g.m, K), device="cuda")
             for cost in COSTS:
-                P, Lp = M.plan(g.m, g.nnz, K, 0, cost, 0)
+                P, Lp = M.plan(g.m, g.nnz, K, DT, cost, 0)
                 cx = torch.empty(P + 1, dtype=torch.int32, device="cuda")
                 cy = torch.empty_like(cx)
                 L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx), _p(cy), s)
 
                 def run():
-                    L.mps_spmm(ctypes.byref(a), _p(B), 0, K, K, _p(C), K, _p(cx), _p(cy), P, 1,
+                    L.mps_spmm(ctypes.byref(a), _p(B), DT, K, K, _p(C), K, _p(cx), _p(cy), P, 1,
                                None, 0, _stream())
                 ms = replay_ms(run)
                 row = {"graph": nm, "type": ty, "n": g.m, "nnz": g.nnz, "K": K, "cost": cost,
@@ -77,7 +80,7 @@ def main():
                     row["writes_atomic"], row["writes_regular"] = int(c[0]), int(c[1])
                     run()
                     torch.cuda.synchronize()
-                    ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B.cpu().numpy())
+                    ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B.float().cpu().numpy())
                     row["parity_ok"] = bool(O.check(C.cpu().numpy(), ref, bnd)["ok"])
                 out.write(json.dumps(row) + "\n")
                 out.flush()
