@@ -116,11 +116,13 @@ Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C
     // rows per instruction mean shorter row-end butterflies and fewer predicated passes
     // per batch; measured on the 22 Table-II graphs (CUDA-graph replay) over 16-B
     // gathers with 16-32 rows per instruction: fp32 K=2/4/8 +4/12/8%, bf16 K=4/8/16
-    // +11/35/16% (profiles/r01/narrow_k/).  MPS_NARROW=0 disables.
+    // +11/35/16% (profiles/r01/narrow_k/; 8 lanes: within 1% except bf16 K=32 +6%).
+    // MPS_NARROW = minimum lanes per row (0 disables).
     int wcap = max_w;
-    const char *en = getenv("MPS_NARROW");
-    if (!en || atoi(en) != 0) {
-        int lim = K / 4 < 1 ? 1 : K / 4;
+    const char *en = getenv("MPS_NARROW");    // minimum lanes per row (default 4; 0: off)
+    const int min_lanes = en ? atoi(en) : 4;
+    if (min_lanes > 0) {
+        int lim = K / min_lanes < 1 ? 1 : K / min_lanes;
         int p2 = 1;
         while (p2 * 2 <= lim) p2 *= 2;
         if (p2 < wcap) wcap = p2;
