@@ -57,6 +57,17 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_UL_DIV
 #define MPS_UL_DIV 1
 #endif
+#ifndef MPS_UMAX
+#define MPS_UMAX 32        // non-zeros per batch (all lane groups) at most
+#endif
+// Gathers per lane per batch in the static instantiation (graphs with < 4 segments per
+// warp: latency-bound kernels of tens of microseconds) when NR >= 2: smaller batches
+// cross fewer row ends.  Table-II graphs: fp32 K=32 +16%, K=64 +8%, bf16 K=64 +7%,
+// K=128 +5%, others within 1% (profiles/r01/batch_size/).  The dynamic instantiation
+// (large graphs) keeps ~4 KB of gathers in flight per warp.
+#ifndef MPS_STATIC_ULCAP
+#define MPS_STATIC_ULCAP 4
+#endif
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
 #endif
@@ -83,7 +94,8 @@ segment_kernel(const SegArgsT<IT> a) {
     constexpr int UL00 = (V * kWords >= 8) ? 4 : ((V * kWords >= 4) ? 8 : 16);
     constexpr int UL0 = (sizeof(TB) == 2 && UL00 / MPS_UL_DIV >= 2) ? UL00 / MPS_UL_DIV
                                                                     : UL00 * (DEEP ? 2 : 1);
-    constexpr int UL = (UL0 * NR > 32) ? (32 / NR > 0 ? 32 / NR : 1) : UL0;
+    constexpr int UL1 = (UL0 * NR > MPS_UMAX) ? (MPS_UMAX / NR > 0 ? MPS_UMAX / NR : 1) : UL0;
+    constexpr int UL = (!DYN && NR >= 2 && UL1 > MPS_STATIC_ULCAP) ? MPS_STATIC_ULCAP : UL1;
     constexpr int U = UL * NR;                           // non-zeros per batch
     static_assert(kCH % U == 0, "chunk must hold whole batches");
 
