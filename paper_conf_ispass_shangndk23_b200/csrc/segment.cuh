@@ -117,6 +117,10 @@ segment_kernel(const SegArgsT<IT> a) {
     }
     mbar_fence_init();
     __syncthreads();
+    // Programmatic dependent launch: this grid may start while the previous kernel of
+    // the stream (the partition / cut-row zeroing) drains; everything above is private
+    // set-up, and nothing it wrote is read before this wait (a no-op without PDL).
+    asm volatile("griddepcontrol.wait;" ::: "memory");
 
     const uint64_t pol_last = a.l2_hints ? policy_evict_last() : policy_evict_normal();
     const uint64_t pol_first = a.l2_hints ? policy_evict_first() : policy_evict_normal();
@@ -566,11 +570,27 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
         arg.claim = base + 2 * (g_claim_next.fetch_add(1u) % kClaimSlots);
         dyn = true;
     }
+    // launched with programmatic stream serialization (PDL): the CTAs may be scheduled
+    // as the previous kernel's CTAs retire, hiding the launch gap (tens of percent of a
+    // small graph's step); griddepcontrol.wait in the kernel keeps the data dependency.
+    // MPS_PDL=0 launches plainly.
+    static const int pdl = [] {
+        const char *e = getenv("MPS_PDL");
+        return e ? atoi(e) : 1;
+    }();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(kBlock);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl ? 1 : 0;
     if (dyn)
-        segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true><<<(unsigned)grid, kBlock, 0, s>>>(arg);
-    else
-        segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false><<<(unsigned)grid, kBlock, 0, s>>>(arg);
-    return cudaGetLastError();
+        return cudaLaunchKernelEx(&cfg, segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>, arg);
+    return cudaLaunchKernelEx(&cfg, segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>, arg);
 }
 
 // (W, V, NR) dispatch.  NR > 1 only with V == 1.
