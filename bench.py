@@ -404,20 +404,23 @@ def main():
             launches_per_step += 4
 
         def step(ev=None):
+            # the stream is looked up per call: under torch.cuda.graph capture the current
+            # stream is the capture stream, and launches elsewhere would not be captured
+            sp = _stream()
             if hot_rows >= 0:              # hub rows of B -> L2 evict_last (recomputed)
                 L.mps_hot_rows(ctypes.byref(a), hot_rows, _p(hot_bm), _p(hot_ws), nbh.value,
-                               s_ptr)
+                               sp)
             if fix != L.MPS_FIXUP_CARRY:   # a2 + zeroing of the cut rows, one launch
                 L.mps_partition_split(_p(A.row_ptr), g.m, g.nnz, P, Lp, _p(cx), _p(cy), _p(C),
-                                      K, K, s_ptr)
+                                      K, K, sp)
             else:
                 L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx),
-                                _p(cy), s_ptr)
+                                _p(cy), sp)
             if ev is not None:
                 ev[0].record(stream)
             L.mps_spmm_segments_hot(ctypes.byref(a), _p(Bd), dt_code, K, K, _p(C), K, _p(cx),
                                     _p(cy), P, fix, _p(hot_bm) if hot_rows >= 0 else None,
-                                    _p(ws), nb.value, s_ptr)
+                                    _p(ws), nb.value, sp)
             if ev is not None:
                 ev[1].record(stream)
         units_nnz = g.nnz
@@ -517,10 +520,19 @@ def main():
 
     run_step = step
     if args.cuda_graph and world == 1:
+        C_eager = C.clone() if world == 1 else None
         cg = torch.cuda.CUDAGraph()
         with torch.cuda.graph(cg):
             step()
         torch.cuda.synchronize(dev)
+        C.fill_(float("nan"))
+        cg.replay()
+        torch.cuda.synchronize(dev)
+        # a replay must reproduce the eager step (an empty capture would leave the NaNs)
+        scale = float(C_eager.abs().max()) if C_eager.numel() else 0.0
+        if not torch.allclose(C, C_eager, rtol=1e-4, atol=1e-5 * scale + 1e-30):
+            raise RuntimeError("CUDA-graph replay does not reproduce the eager step")
+        del C_eager
 
         def run_step(ev=None):            # events cannot split a replay: time the graph
             if ev is not None:

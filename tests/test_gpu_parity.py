@@ -646,3 +646,25 @@ def test_products_full_size_k128():
     g = G.workload("products")
     _sampled_check(g, 128, "atomic")
     _sampled_check(g, 128, "atomic", dtype=torch.bfloat16)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("wl,K", [("cora", 16), ("rmat", 64)])
+def test_bench_cuda_graph_replays_the_step(wl, K):
+    """bench.py --cuda-graph: the captured graph must hold the step's launches (the bench
+    itself replays once against the eager result and raises on a mismatch), and a replay
+    cannot be faster than the segment kernel's share of the eager step."""
+    import json, os, subprocess, sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    base = [sys.executable, os.path.join(root, "bench.py"), "--workload", wl, "--K", str(K),
+            "--steps", "5", "--warmup", "3", "--e2e-steps", "0", "--no-cpu-baseline",
+            "--no-cusparse", "--no-l2-probe"]
+    lines = {}
+    for mode in ("eager", "graph"):
+        cmd = base + (["--cuda-graph"] if mode == "graph" else [])
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=root)
+        assert r.returncode == 0, r.stderr[-2000:]
+        lines[mode] = json.loads([ln for ln in r.stdout.splitlines() if ln.startswith("{")][-1])
+    assert lines["graph"]["config"]["cuda_graph"] is True
+    # the eager step's segment kernel alone bounds the graph replay from below
+    assert lines["graph"]["ms_per_step"] >= 0.5 * lines["eager"]["segment_ms"]
