@@ -88,7 +88,9 @@ partition_kernel(const IT *__restrict__ rp, int64_t m, int64_t nnz, int64_t d0,
         cy[p] = (IT)y;
     }
     if (zero_C == nullptr && tail == nullptr) return;  // uniform across the grid
-    const bool inside = valid && x < m && y > (int64_t)__ldg(rp + x);
+    // x lies in [xlo, xhi]: rp[x] comes from the staged window when there is one
+    const bool inside = valid && x < m &&
+                        y > (staged ? (int64_t)s_rp[x - xlo] : (int64_t)__ldg(rp + x));
     unsigned todo = __ballot_sync(0xffffffffu, inside);
     while (todo) {
         const int src = __ffs(todo) - 1;
