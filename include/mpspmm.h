@@ -12,7 +12,13 @@
  *    returns an mps_status; mps_last_error() gives a thread-local detail string.
  *  - Ownership: the caller allocates and frees every buffer (A, B, C, coordinates,
  *    workspace, tails).  The library keeps no global state and allocates nothing
- *    persistent; all functions are reentrant.
+ *    persistent; all functions are reentrant.  Everything a launch needs beyond its
+ *    arguments lives in the caller's workspace -- including the counters from which
+ *    the segment kernel's warps claim segments (one 32-bit word per column tile,
+ *    zeroed on the stream by the call that uses them) -- so two calls (or two captured
+ *    CUDA graphs) running concurrently must use different workspaces, and never
+ *    interfere otherwise.  Host-side caches are per device and hold only occupancy
+ *    and attribute queries.
  *  - Pointers are DEVICE pointers unless the parameter name ends in _host.
  *  - Streams: every device call is asynchronous on `stream` (a cudaStream_t passed
  *    as void*; NULL = the legacy default stream).  Only mps_validate_csr
@@ -112,7 +118,8 @@ mps_status mps_partition_split(const int32_t *row_ptr, int64_t m, int64_t nnz,
  * are stored, split rows are zeroed first or stored by the carry pass, empty rows
  * get 0).  B: n rows, leading dimension ldb elements (b_dtype); C: m rows, leading
  * dimension ldc floats.  workspace: caller-owned device memory of at least
- * mps_spmm_workspace_bytes(...) bytes (may be NULL when that is 0).              */
+ * mps_spmm_workspace_bytes(...) bytes (>= 256: the segment-claim counters, then the
+ * carry records in carry mode); its content on entry does not matter.           */
 mps_status mps_spmm_workspace_bytes(const mps_csr *A, int32_t K, int32_t b_dtype,
                                     int64_t num_parts, int32_t fixup, size_t *bytes);
 mps_status mps_spmm(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb, int32_t K,
@@ -124,7 +131,9 @@ mps_status mps_spmm(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ld
  * mps_zero_split_rows zeroes the rows cut by a boundary of the schedule (x_p < m,
  * y_p > row_ptr[x_p]; the atomic fix-up's precondition, reading R10);
  * mps_spmm_segments runs a3 (+ the a4 carry reduction) and, in atomic mode,
- * REQUIRES that mps_zero_split_rows ran earlier on the same C and schedule.       */
+ * REQUIRES that mps_zero_split_rows ran earlier on the same C and schedule.  Its
+ * workspace is sized by mps_spmm_workspace_bytes; for long schedules it zeroes the
+ * claim counters there with one cudaMemsetAsync before the segment kernel.       */
 mps_status mps_zero_split_rows(const mps_csr *A, const int32_t *coord_x, const int32_t *coord_y,
                                int64_t num_parts, float *C, int64_t ldc, int32_t K,
                                void *stream);
@@ -184,7 +193,13 @@ mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, 
  * and copies C device->host, all enqueued on `stream` (pinned host memory gives
  * true async copies).  A_host holds HOST pointers.  device_workspace: caller-owned
  * device memory of mps_spmm_host_workspace_bytes(...) bytes.  The caller
- * synchronises the stream before reading C_host.                                 */
+ * synchronises the stream before reading C_host.  Only the K valid columns of each
+ * row are copied: with ldb > K or ldc > K the padding of B_host is never read and
+ * the padding of C_host never written.  In atomic mode the call pipelines the H2D of
+ * A (merge-path chunks) with the segment kernels and the D2H of finished rows on two
+ * streams it creates for the call and releases when the call's work completes; the
+ * whole call is ordered after earlier work on `stream` and later work on `stream`
+ * waits for it.                                                                  */
 mps_status mps_spmm_host_workspace_bytes(const mps_csr *A_host, int32_t K, int32_t b_dtype,
                                          int64_t ldb, int64_t ldc, int64_t items_per_part,
                                          int64_t min_parts, int32_t fixup, size_t *bytes);

@@ -91,8 +91,8 @@ def plan(m, nnz, K, b_dtype=L.MPS_DT_F32, items_per_part=0, min_parts=0, wide=Fa
 def partition(A: CSR, num_parts, items_per_part, diag_begin=0, diag_end=None, stream=None):
     """a2: coordinates (x_p, y_p), p = 0..P, of the merge-path diagonals (Alg. 1 l.4-7)."""
     diag_end = A.m + A.nnz if diag_end is None else diag_end
-    cx = torch.empty(num_parts + 1, dtype=torch.int32, device=A.device)
-    cy = torch.empty(num_parts + 1, dtype=A.row_ptr.dtype, device=A.device)
+    cx = _keep(torch.empty(num_parts + 1, dtype=torch.int32, device=A.device), stream)
+    cy = _keep(torch.empty(num_parts + 1, dtype=A.row_ptr.dtype, device=A.device), stream)
     f = L.mps_partition64 if A.wide else L.mps_partition
     f(_p(A.row_ptr), A.m, A.nnz, diag_begin, diag_end, num_parts, items_per_part,
       _p(cx), _p(cy), _stream(stream))
@@ -115,8 +115,18 @@ class Schedule:
         return cls(P, Lp, cx, cy)
 
 
-def _ws(nbytes, device):
-    return torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=device)
+def _ws(nbytes, device, stream=None):
+    """Workspace for one call.  Allocated on the current stream; when the call runs on
+    another ``stream`` the allocation is recorded there, so the caching allocator does
+    not hand the memory out again before that stream's kernels are done with it."""
+    t = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=device)
+    return _keep(t, stream)
+
+
+def _keep(t, stream):
+    if stream is not None and t is not None and stream != torch.cuda.current_stream(t.device):
+        t.record_stream(stream)
+    return t
 
 
 EPILOGUE = {"none": L.MPS_EPI_NONE, "relu": L.MPS_EPI_RELU}
@@ -133,7 +143,10 @@ def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomi
     assert B.dim() == 2 and B.stride(1) == 1 and B.device == A.device
     K = B.shape[1]
     dt = _dtype_code(B)
-    C = torch.empty((A.m, K), dtype=torch.float32, device=A.device) if out is None else out
+    C = torch.empty((A.m, K), dtype=torch.float32, device=A.device) if out is None \
+        else out
+    if out is None:
+        _keep(C, stream)
     assert C.stride(1) == 1 and C.shape == (A.m, K)
     a = A.struct()
     nb = ctypes.c_size_t()
@@ -142,28 +155,28 @@ def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomi
         if schedule is not None:
             L.mps_spmm64_workspace_bytes(ctypes.byref(a), K, dt, schedule.num_parts,
                                          _fix(fixup), ctypes.byref(nb))
-            ws = _ws(nb.value, A.device)
+            ws = _ws(nb.value, A.device, stream)
             L.mps_spmm64(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
                          _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts,
                          _fix(fixup), EPILOGUE[epilogue], _p(ws), nb.value, st)
         else:
             L.mps_spmm64_online_workspace_bytes(ctypes.byref(a), K, dt, items_per_part,
                                                 min_parts, _fix(fixup), ctypes.byref(nb))
-            ws = _ws(nb.value, A.device)
+            ws = _ws(nb.value, A.device, stream)
             L.mps_spmm64_online(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
                                 items_per_part, min_parts, _fix(fixup), EPILOGUE[epilogue],
                                 _p(ws), nb.value, st)
     elif schedule is not None:
         L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt, schedule.num_parts, _fix(fixup),
                                    ctypes.byref(nb))
-        ws = _ws(nb.value, A.device)
+        ws = _ws(nb.value, A.device, stream)
         L.mps_spmm_ex(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
                       _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts,
                       _fix(fixup), EPILOGUE[epilogue], None, _p(ws), nb.value, st)
     else:
         L.mps_spmm_online_workspace_bytes(ctypes.byref(a), K, dt, items_per_part, min_parts,
                                           _fix(fixup), ctypes.byref(nb))
-        ws = _ws(nb.value, A.device)
+        ws = _ws(nb.value, A.device, stream)
         L.mps_spmm_online_ex(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
                              items_per_part, min_parts, _fix(fixup), EPILOGUE[epilogue],
                              _p(ws), nb.value, st)
@@ -220,10 +233,13 @@ def xw_bf16(X: torch.Tensor, Wt: torch.Tensor, out: torch.Tensor | None = None, 
             return t
         buf = torch.zeros((t.shape[0], -(-t.shape[1] // 8) * 8), dtype=t.dtype, device=t.device)
         buf[:, : t.shape[1]] = t
-        return buf[:, : t.shape[1]]
+        if stream is not None:       # the staging copy must be complete before `stream` reads it
+            stream.wait_stream(torch.cuda.current_stream(t.device))
+        return _keep(buf, stream)[:, : t.shape[1]]
     X, Wt = tma_ready(X), tma_ready(Wt)
     N = Wt.shape[0]
-    B = torch.empty((n, N), dtype=torch.bfloat16, device=X.device) if out is None else out
+    B = _keep(torch.empty((n, N), dtype=torch.bfloat16, device=X.device), stream) \
+        if out is None else out
     L.mps_xw_bf16(_p(X), n, F, X.stride(0), _p(Wt), N, Wt.stride(0), _p(B), B.stride(0),
                   _stream(stream))
     return B
@@ -288,10 +304,13 @@ def host_workspace_bytes(row_ptr, col_idx, val, n_cols, B_host, C_host, items_pe
 
 def write_stats(A: CSR, schedule: Schedule, stream=None):
     """Fig. 5 statistic: (#atomic row updates, #regular row stores) under Alg. 2."""
-    cnt = torch.empty(2, dtype=torch.int64, device=A.device)
+    cnt = _keep(torch.empty(2, dtype=torch.int64, device=A.device), stream)
     a = A.struct()
-    (L.mps_write_stats64 if A.wide else L.mps_write_stats)(ctypes.byref(a), _p(schedule.coord_x), _p(schedule.coord_y),
-                      schedule.num_parts, _p(cnt), _stream(stream))
+    (L.mps_write_stats64 if A.wide else L.mps_write_stats)(
+        ctypes.byref(a), _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts,
+        _p(cnt), _stream(stream))
+    if stream is not None:          # the counts are read on the host: wait for `stream`
+        stream.synchronize()
     c = cnt.cpu()
     return int(c[0]), int(c[1])
 
@@ -302,3 +321,84 @@ def validate_csr(A: CSR, stream=None) -> int:
     bad = ctypes.c_int64()
     (L.mps_validate_csr64 if A.wide else L.mps_validate_csr)(ctypes.byref(a), ctypes.byref(bad), _stream(stream))
     return bad.value
+
+
+class OnlineStep:
+    """One online MergePath-SpMM step as two library calls, for callers that time the
+    segment kernel on its own (bench.py's path of record; the full-size parity tests run
+    exactly this):
+
+      a1 ``mps_plan`` (host, once) ->
+      a2 + a4 zeroing: ``mps_partition_split`` (atomic) / ``mps_partition`` (carry) ->
+      a3 (+ a4 carry reduction): ``mps_spmm_segments_hot`` (dynamic segment claims from
+      counters in ``ws``, programmatic dependent launch after the partition kernel).
+
+    ``mps_spmm_online`` issues the same kernels in one call.  Buffers (coordinates, C,
+    workspace, optional hot-row bitmap) are allocated once and reused by every call, so
+    a call can be captured in a CUDA graph.  ``events``: (ev_after_partition,
+    ev_after_segments) recorded on the launching stream."""
+
+    def __init__(self, A: CSR, K: int, b_dtype=torch.float32, fixup="atomic",
+                 items_per_part=0, min_parts=0, hot="auto", out: torch.Tensor | None = None):
+        assert not A.wide, "OnlineStep: int32 indices (mps_csr)"
+        self.A, self.K, self.fixup = A, K, _fix(fixup)
+        self.dt = L.MPS_DT_BF16 if b_dtype == torch.bfloat16 else L.MPS_DT_F32
+        self.a = A.struct()
+        self.P, self.L = plan(A.m, A.nnz, K, self.dt, items_per_part, min_parts)
+        dev = A.device
+        self.cx = torch.empty(self.P + 1, dtype=torch.int32, device=dev)
+        self.cy = torch.empty(self.P + 1, dtype=torch.int32, device=dev)
+        self.C = torch.empty((A.m, K), dtype=torch.float32, device=dev) if out is None else out
+        assert self.C.stride(1) == 1 and self.C.shape == (A.m, K)
+        nb = ctypes.c_size_t()
+        L.mps_spmm_workspace_bytes(ctypes.byref(self.a), K, self.dt, self.P, self.fixup,
+                                   ctypes.byref(nb))
+        self.ws_bytes = nb.value
+        self.ws = _ws(nb.value, dev)
+        hr = ctypes.c_int64(-1)
+        if hot == "auto":
+            L.mps_hot_budget_rows(ctypes.byref(self.a), K, self.dt, ctypes.byref(hr))
+        self.hot_rows = hr.value
+        self.hot_bm = None
+        if self.hot_rows >= 0:
+            nbh = ctypes.c_size_t()
+            L.mps_hot_rows_workspace_bytes(A.n, ctypes.byref(nbh))
+            self.hot_ws_bytes = nbh.value
+            self.hot_ws = _ws(nbh.value, dev)
+            self.hot_bm = torch.empty((A.n + 31) // 32, dtype=torch.int32, device=dev)
+
+    def __call__(self, B: torch.Tensor, events=None, stream=None):
+        assert B.dim() == 2 and B.stride(1) == 1 and B.shape[1] == self.K
+        assert _dtype_code(B) == self.dt
+        s = _stream(stream)           # looked up per call: CUDA-graph capture streams
+        A, a = self.A, ctypes.byref(self.a)
+        if self.hot_bm is not None:   # hub rows of B -> L2 evict_last (recomputed per call)
+            L.mps_hot_rows(a, self.hot_rows, _p(self.hot_bm), _p(self.hot_ws),
+                           self.hot_ws_bytes, s)
+        if self.fixup != L.MPS_FIXUP_CARRY:      # a2 + zeroing of the cut rows, one launch
+            L.mps_partition_split(_p(A.row_ptr), A.m, A.nnz, self.P, self.L, _p(self.cx),
+                                  _p(self.cy), _p(self.C), self.C.stride(0), self.K, s)
+        else:
+            L.mps_partition(_p(A.row_ptr), A.m, A.nnz, 0, A.m + A.nnz, self.P, self.L,
+                            _p(self.cx), _p(self.cy), s)
+        st = stream or torch.cuda.current_stream(A.device)
+        if events is not None:
+            events[0].record(st)
+        L.mps_spmm_segments_hot(a, _p(B), self.dt, B.stride(0), self.K, _p(self.C),
+                                self.C.stride(0), _p(self.cx), _p(self.cy), self.P, self.fixup,
+                                _p(self.hot_bm), _p(self.ws), self.ws_bytes, s)
+        if events is not None:
+            events[1].record(st)
+        return self.C
+
+    def launches(self, l2_bytes: int) -> int:
+        """Library kernels (and memsets) one call enqueues."""
+        eb = 2 if self.dt == L.MPS_DT_BF16 else 4
+        tile = 512 if eb == 4 else 1024
+        if self.A.n * self.K * eb > 0.5 * l2_bytes:
+            tile = min(tile, 256 // eb)
+        tiles = -(-self.K // min(self.K, tile)) if self.K else 0
+        n = 1 + tiles * (2 if self.fixup == L.MPS_FIXUP_CARRY else 1)
+        if self.hot_bm is not None:
+            n += 4
+        return n

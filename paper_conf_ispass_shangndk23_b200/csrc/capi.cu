@@ -5,7 +5,6 @@
 #include <cstdarg>
 #include <cstdlib>
 #include <type_traits>
-#include <mutex>
 #include <vector>
 
 #include <cuda.h>
@@ -212,6 +211,17 @@ size_t carry_bytes(int64_t P, int32_t K, const Vec &v) {
     return (size_t)P * 2 * (size_t)carry_kpad(K, v) * sizeof(float);
 }
 
+// Dynamic segment claims: one 32-bit counter per column tile, in the caller's workspace
+// (no library state: every workspace, and so every captured CUDA graph, owns its
+// counters).  Sized for the worst case of one column per tile.
+size_t claim_bytes(int32_t K) { return align_up((size_t)(K > 0 ? K : 1) * 4, 256); }
+int32_t num_tiles(int32_t K, const Vec &v) { return K > 0 ? (K + v.tile - 1) / v.tile : 0; }
+// claim counters a kernel preceding the segment kernel can zero (one per thread of a CTA)
+int32_t zeroable_claims(int32_t K, const Vec &v) {
+    const int32_t t = num_tiles(K, v);
+    return t <= mps::kBlock ? t : 0;
+}
+
 int resolve_fix(int32_t fixup) { return fixup == MPS_FIXUP_CARRY ? mps::FIX_CARRY : mps::FIX_ATOMIC; }
 
 // host coordinate of diagonal d (shard bounds): x = max{x : x + rp[x] <= d}
@@ -227,10 +237,17 @@ int64_t host_diag_x(const IT *rp, int64_t m, int64_t nnz, int64_t d) {
 }
 
 // Run a3 (+ a4 carry reduction) over all column tiles for a ready schedule.
+// claims: the per-tile claim counters (workspace; NULL: static segment assignment);
+// claims_zeroed: a kernel earlier on the stream already zeroed them, else they are
+// zeroed here when the schedule is long enough for dynamic claims.
 template <typename IT>
 mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec &v, int fix,
-                        void *workspace, cudaStream_t s) {
+                        void *workspace, unsigned *claims, bool claims_zeroed,
+                        cudaStream_t s) {
     const int eb = elt_bytes(dt);
+    if (claims && !claims_zeroed && base.P >= mps::seg_dynamic_min_parts())
+        MPS_CUDA(cudaMemsetAsync(claims, 0, (size_t)num_tiles(K, v) * 4, s), "zero claims");
+    if (claims && !claims_zeroed && base.P < mps::seg_dynamic_min_parts()) claims = nullptr;
     for (int32_t c0 = 0; c0 < K; c0 += v.tile) {
         mps::SegArgsT<IT> a = base;
         // the tail exchange rides on the launch that finalises the tail: the last tile's
@@ -243,6 +260,7 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
         a.tail = base.tail ? base.tail + c0 : nullptr;
         a.rec = (float *)workspace;
         a.kpad = (int32_t)carry_kpad(K, v);
+        a.claim = claims ? claims + c0 / v.tile : nullptr;
         // TMA staging needs col and val equally aligned modulo 16 B
         a.direct = ((((uintptr_t)base.col) ^ ((uintptr_t)base.val)) & 15u) != 0;
         static const int hints = [] {
@@ -282,7 +300,7 @@ int num_sms() {
 
 extern "C" {
 
-int mps_abi_version(void) { return 1; }
+int mps_abi_version(void) { return 2; }  // 2: claim counters in the workspace
 
 const char *mps_status_string(mps_status s) {
     switch (s) {
@@ -336,7 +354,7 @@ static mps_status partition_impl(const IT *row_ptr, int64_t m, int64_t nnz, int6
     if (!row_ptr || !coord_x || !coord_y) return fail(MPS_ERR_INVALID, "NULL pointer");
     MPS_CUDA(mps::launch_partition<IT>(row_ptr, m, nnz, diag_begin, diag_end - diag_begin,
                                        num_parts, items_per_part, coord_x, coord_y, nullptr, 0, 0,
-                                       0, -1, nullptr, (cudaStream_t)stream),
+                                       0, -1, nullptr, nullptr, 0, (cudaStream_t)stream),
              "partition kernel");
     return MPS_OK;
 }
@@ -380,7 +398,7 @@ mps_status mps_partition_split(const int32_t *row_ptr, int64_t m, int64_t nnz,
         return fail(MPS_ERR_INVALID, "NULL pointer");
     MPS_CUDA(mps::launch_partition(row_ptr, m, nnz, 0, m + nnz, num_parts, items_per_part, coord_x,
                                    coord_y, K > 0 ? C : nullptr, ldc, 0, K, -1, nullptr,
-                                   (cudaStream_t)stream),
+                                   nullptr, 0, (cudaStream_t)stream),
              "partition kernel");
     return MPS_OK;
 }
@@ -410,20 +428,22 @@ mps_status spmm_ws_impl(const CSR *A, int32_t K, int32_t b_dtype, int64_t num_pa
                       ? (carry_bytes(num_parts, K, v) > carry_bytes(num_parts, K, vmin)
                              ? carry_bytes(num_parts, K, v) : carry_bytes(num_parts, K, vmin))
                       : 0;
-    *bytes = need;
+    *bytes = claim_bytes(K) + need;   // [claim counters][carry records]
     return MPS_OK;
 }
 
 template <typename CSR>
 mps_status zero_split_impl(const CSR *A, const int32_t *coord_x, const idx_t<CSR> *coord_y,
-                           int64_t num_parts, float *C, int64_t ldc, int32_t K, void *stream) {
+                           int64_t num_parts, float *C, int64_t ldc, int32_t K, void *stream,
+                           unsigned *claims = nullptr, int32_t nclaims = 0) {
     mps_status st = check_csr(A);
     if (st) return st;
     if (num_parts < 1 || K < 0 || (K > 0 && ldc < K)) return fail(MPS_ERR_INVALID, "bad arguments");
     if (K == 0 || A->m == 0) return MPS_OK;
     if (!coord_x || !coord_y || !C) return fail(MPS_ERR_INVALID, "NULL pointer");
     MPS_CUDA(mps::launch_zero_split(A->row_ptr, (int32_t)A->m, coord_x, coord_y, num_parts, C,
-                                    ldc, 0, K, -1, nullptr, (cudaStream_t)stream),
+                                    ldc, 0, K, -1, nullptr, claims, nclaims,
+                                    (cudaStream_t)stream),
              "zero split rows");
     return MPS_OK;
 }
@@ -433,7 +453,7 @@ mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t l
                          float *C, int64_t ldc, const int32_t *coord_x,
                          const idx_t<CSR> *coord_y, int64_t num_parts, int32_t fixup,
                          const uint32_t *hot_bitmap, int32_t relu, void *workspace,
-                         size_t workspace_bytes, void *stream) {
+                         size_t workspace_bytes, void *stream, bool claims_zeroed = false) {
     mps_status st = check_csr(A);
     if (st) return st;
     if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
@@ -442,10 +462,10 @@ mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t l
     if (!coord_x || !coord_y) return fail(MPS_ERR_INVALID, "NULL coordinates");
     const int fix = resolve_fix(fixup);
     const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n, A->m, A->nnz);
-    if (fix == mps::FIX_CARRY && workspace_bytes < carry_bytes(num_parts, K, v))
-        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes,
-                    carry_bytes(num_parts, K, v));
-    if (fix == mps::FIX_CARRY && !workspace) return fail(MPS_ERR_WORKSPACE, "workspace NULL");
+    // workspace: [claim counters][carry records (carry mode)]
+    const size_t need = claim_bytes(K) + (fix == mps::FIX_CARRY ? carry_bytes(num_parts, K, v) : 0);
+    if (!workspace || workspace_bytes < need)
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
     mps::SegArgsT<idx_t<CSR>> a{};
     a.rp = A->row_ptr;
     a.col = A->col_idx;
@@ -464,7 +484,8 @@ mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t l
     a.nnz_end = A->nnz;
     a.hot = hot_bitmap;
     a.relu = relu;
-    return run_segments(a, b_dtype, K, v, fix, workspace, (cudaStream_t)stream);
+    return run_segments(a, b_dtype, K, v, fix, (char *)workspace + claim_bytes(K),
+                        (unsigned *)workspace, claims_zeroed, (cudaStream_t)stream);
 }
 
 template <typename CSR>
@@ -481,8 +502,16 @@ mps_status spmm_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t ld
         if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
         if (num_parts < 1) return fail(MPS_ERR_INVALID, "num_parts < 1");
         if (K == 0 || A->m == 0) return MPS_OK;
-        if ((st = zero_split_impl(A, coord_x, coord_y, num_parts, C, ldc, K, stream)))
+        const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n, A->m, A->nnz);
+        const int32_t nz = zeroable_claims(K, v);
+        if (!workspace || workspace_bytes < claim_bytes(K))
+            return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, claim_bytes(K));
+        if ((st = zero_split_impl(A, coord_x, coord_y, num_parts, C, ldc, K, stream,
+                                  (unsigned *)workspace, nz)))
             return st;
+        return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                             hot_bitmap, epilogue == MPS_EPI_RELU, workspace, workspace_bytes,
+                             stream, nz > 0);
     }
     return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
                          hot_bitmap, epilogue == MPS_EPI_RELU, workspace, workspace_bytes,
@@ -526,10 +555,12 @@ int64_t hot_budget_rows(int64_t n, int32_t K, int32_t dt) {
     return (int64_t)(frac * (double)l2_bytes() / row);
 }
 
-// online workspace: coord_x int32[P+1], coord_y IT[P+1], carry records, hot-row scratch
+// online workspace: coord_x int32[P+1], coord_y IT[P+1], claim counters, carry records,
+// hot-row scratch
 size_t online_bytes(int64_t P, int32_t K, const Vec &v, int fix, int64_t n = 0,
                     size_t ysize = 4) {
-    size_t b = align_up((size_t)(P + 1) * 4, 256) + align_up((size_t)(P + 1) * ysize, 256);
+    size_t b = align_up((size_t)(P + 1) * 4, 256) + align_up((size_t)(P + 1) * ysize, 256) +
+               claim_bytes(K);
     if (fix == mps::FIX_CARRY) b += carry_bytes(P, K, v);
     if (n > 0) b += hot_bitmap_bytes(n) + hot_scratch_bytes(n);
     return b;
@@ -585,7 +616,9 @@ mps_status online_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t 
     const size_t yb = align_up((size_t)(P + 1) * sizeof(IT), 256);
     int32_t *cx = (int32_t *)workspace;
     IT *cy = (IT *)((char *)workspace + xb);
-    void *rec = (char *)workspace + xb + yb;
+    unsigned *claims = (unsigned *)((char *)workspace + xb + yb);
+    void *rec = (char *)workspace + xb + yb + claim_bytes(K);
+    const int32_t nz = zeroable_claims(K, v);
     uint32_t *bitmap = nullptr;
     if (nh > 0) {
         char *hb = (char *)workspace + online_bytes(P, K, v, fix, 0, sizeof(IT));
@@ -596,7 +629,7 @@ mps_status online_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t 
     }
     MPS_CUDA(mps::launch_partition<IT>(A->row_ptr, A->m, A->nnz, 0, A->m + A->nnz, P, L, cx, cy,
                                        fix == mps::FIX_ATOMIC ? C : nullptr, ldc, 0, K, -1,
-                                       nullptr, s),
+                                       nullptr, claims, nz, s),
              "partition kernel");
     mps::SegArgsT<IT> a{};
     a.rp = A->row_ptr;
@@ -616,7 +649,7 @@ mps_status online_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t 
     a.nnz_end = A->nnz;
     a.hot = bitmap;
     a.relu = epilogue == MPS_EPI_RELU;
-    return run_segments(a, b_dtype, K, v, fix, rec, s);
+    return run_segments(a, b_dtype, K, v, fix, rec, claims, nz > 0, s);
 }
 
 template <typename CSR>
@@ -827,26 +860,23 @@ mps_status mps_spmm_host_workspace_bytes(const mps_csr *A_host, int32_t K, int32
 // at x_{c+1} belongs to the next range.  One partition (+ cut-row zeroing) launch over
 // all P segments serves every chunk, so the result is the one mps_spmm_online gives.
 namespace {
+// The pipelined host call's two auxiliary streams (compute, D2H) are created per call and
+// released when the call's work completes: the library keeps no streams between calls.
 struct AuxStreams {
     cudaStream_t comp = nullptr, d2h = nullptr;
-};
-AuxStreams aux_streams() {
-    static AuxStreams cache[64];
-    static std::mutex mu;
-    int dev = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return AuxStreams{};
-    std::lock_guard<std::mutex> lock(mu);
-    if (!cache[dev].comp) {
-        cudaStream_t a = nullptr, b = nullptr;
-        if (cudaStreamCreateWithFlags(&a, cudaStreamNonBlocking) != cudaSuccess) return AuxStreams{};
-        if (cudaStreamCreateWithFlags(&b, cudaStreamNonBlocking) != cudaSuccess) {
-            cudaStreamDestroy(a);
-            return AuxStreams{};
-        }
-        cache[dev].d2h = b;
-        cache[dev].comp = a;
+    ~AuxStreams() {
+        if (comp) cudaStreamDestroy(comp);   // deferred by the runtime until the work is done
+        if (d2h) cudaStreamDestroy(d2h);
     }
-    return cache[dev];
+};
+
+// rows x width bytes between pitched buffers: only the K valid columns of a strided
+// (ld > K) host matrix are read or written, never its padding
+cudaError_t copy_rows(void *dst, const void *src, size_t pitch, size_t width, size_t rows,
+                      cudaMemcpyKind kind, cudaStream_t s) {
+    if (rows == 0 || width == 0) return cudaSuccess;
+    if (pitch == width) return cudaMemcpyAsync(dst, src, rows * width, kind, s);
+    return cudaMemcpy2DAsync(dst, pitch, src, pitch, width, rows, kind, s);
 }
 
 bool getenv_flag(const char *name) {
@@ -865,8 +895,10 @@ static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int3
                                  int64_t ldb, int32_t K, float *C_host, int64_t ldc,
                                  int64_t P, int64_t L, const Vec &v, const HostLayout &h,
                                  char *w, cudaStream_t s) {
-    const AuxStreams ax = aux_streams();
-    if (!ax.comp) return fail(MPS_ERR_CUDA, "auxiliary streams");
+    AuxStreams ax;
+    if (cudaStreamCreateWithFlags(&ax.comp, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&ax.d2h, cudaStreamNonBlocking) != cudaSuccess)
+        return fail(MPS_ERR_CUDA, "auxiliary streams");
     const int64_t m = A_host->m, nnz = A_host->nnz, M = m + nnz;
     int64_t nc = (nnz * 8 + host_chunk_bytes() - 1) / host_chunk_bytes();
     if (nc < 1) nc = 1;
@@ -880,6 +912,7 @@ static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int3
         yc[c] = d - xc[c];
     }
     const size_t bbytes = (size_t)A_host->n * (size_t)ldb * elt_bytes(b_dtype);
+    const size_t brow = (size_t)ldb * elt_bytes(b_dtype), bwidth = (size_t)K * elt_bytes(b_dtype);
     int32_t *rp = (int32_t *)(w + h.rp);
     int32_t *ci = (int32_t *)(w + h.ci);
     float *va = (float *)(w + h.val);
@@ -905,7 +938,9 @@ static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int3
     chk(cudaMemcpyAsync(rp, A_host->row_ptr, (size_t)(m + 1) * 4, cudaMemcpyHostToDevice, s),
         "H2D row_ptr");
     chk(cudaEventRecord(ev_rp, s), "event");
-    if (bbytes) chk(cudaMemcpyAsync(w + h.B, B_host, bbytes, cudaMemcpyHostToDevice, s), "H2D B");
+    if (bbytes)
+        chk(copy_rows(w + h.B, B_host, brow, bwidth, (size_t)A_host->n, cudaMemcpyHostToDevice, s),
+            "H2D B");
     chk(cudaEventRecord(ev_B, s), "event");
     for (int64_t c = 0; c < nc && st == MPS_OK; ++c) {
         const size_t n = (size_t)(yc[c + 1] - yc[c]) * 4;
@@ -921,7 +956,7 @@ static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int3
     chk(cudaStreamWaitEvent(ax.comp, ev_rp, 0), "wait");
     if (st == MPS_OK)
         chk(mps::launch_partition<int32_t>(rp, m, nnz, 0, M, P, L, cx, cy, C, ldc, 0, K, -1,
-                                           nullptr, ax.comp), "partition kernel");
+                                           nullptr, nullptr, 0, ax.comp), "partition kernel");
     chk(cudaStreamWaitEvent(ax.comp, ev_B, 0), "wait");
     for (int64_t c = 0; c < nc && st == MPS_OK; ++c) {
         chk(cudaStreamWaitEvent(ax.comp, ev_A[c], 0), "wait");
@@ -944,7 +979,9 @@ static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int3
             a.nnz_end = nnz;
             a.hot = nullptr;
             a.relu = 0;
-            st = run_segments(a, b_dtype, K, v, mps::FIX_ATOMIC, nullptr, ax.comp);
+            // static segment assignment: the chunks' launches would each need their
+            // own claim counters; this path is bound by the H2D copies anyway
+            st = run_segments(a, b_dtype, K, v, mps::FIX_ATOMIC, nullptr, nullptr, true, ax.comp);
         }
         chk(cudaEventRecord(ev_done[c], ax.comp), "event");
     }
@@ -953,8 +990,8 @@ static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int3
         const int64_t r0 = xc[c], r1 = (c + 1 == nc) ? m : xc[c + 1];
         chk(cudaStreamWaitEvent(ax.d2h, ev_done[c], 0), "wait");
         if (r1 > r0)
-            chk(cudaMemcpyAsync(C_host + r0 * ldc, C + r0 * ldc, (size_t)(r1 - r0) * ldc * 4,
-                                cudaMemcpyDeviceToHost, ax.d2h), "D2H C");
+            chk(copy_rows(C_host + r0 * ldc, C + r0 * ldc, (size_t)ldc * 4, (size_t)K * 4,
+                          (size_t)(r1 - r0), cudaMemcpyDeviceToHost, ax.d2h), "D2H C");
     }
     // join: the caller's stream sees the whole call
     chk(cudaEventRecord(ev_end, ax.d2h), "event");
@@ -999,7 +1036,10 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
         MPS_CUDA(cudaMemcpyAsync(w + h.val, A_host->val, (size_t)A_host->nnz * 4,
                                  cudaMemcpyHostToDevice, s), "H2D val");
     }
-    if (bbytes) MPS_CUDA(cudaMemcpyAsync(w + h.B, B_host, bbytes, cudaMemcpyHostToDevice, s), "H2D B");
+    if (bbytes)
+        MPS_CUDA(copy_rows(w + h.B, B_host, (size_t)ldb * elt_bytes(b_dtype),
+                           (size_t)K * elt_bytes(b_dtype), (size_t)A_host->n,
+                           cudaMemcpyHostToDevice, s), "H2D B");
     mps_csr Ad = *A_host;
     Ad.row_ptr = (const int32_t *)(w + h.rp);
     Ad.col_idx = (const int32_t *)(w + h.ci);
@@ -1007,8 +1047,8 @@ mps_status mps_spmm_host(const mps_csr *A_host, const void *B_host, int32_t b_dt
     if ((st = mps_spmm_online(&Ad, w + h.B, b_dtype, ldb, K, (float *)(w + h.C), ldc,
                               items_per_part, min_parts, fixup, w + h.ws, online, stream)))
         return st;
-    MPS_CUDA(cudaMemcpyAsync(C_host, w + h.C, (size_t)A_host->m * (size_t)ldc * 4,
-                             cudaMemcpyDeviceToHost, s), "D2H C");
+    MPS_CUDA(copy_rows(C_host, w + h.C, (size_t)ldc * 4, (size_t)K * 4, (size_t)A_host->m,
+                       cudaMemcpyDeviceToHost, s), "D2H C");
     return MPS_OK;
 }
 
@@ -1048,12 +1088,15 @@ mps_status mps_spmm_host_dense(const mps_csr *A, const void *B_host, int32_t b_d
     char *Bd = w;
     float *Cd = (float *)(w + align_up(bbytes, 256));
     char *ws = (char *)Cd + align_up((size_t)A->m * (size_t)ldc * 4, 256);
-    if (bbytes) MPS_CUDA(cudaMemcpyAsync(Bd, B_host, bbytes, cudaMemcpyHostToDevice, s), "H2D B");
+    if (bbytes)
+        MPS_CUDA(copy_rows(Bd, B_host, (size_t)ldb * elt_bytes(b_dtype),
+                           (size_t)K * elt_bytes(b_dtype), (size_t)A->n, cudaMemcpyHostToDevice,
+                           s), "H2D B");
     if ((st = mps_spmm_online(A, Bd, b_dtype, ldb, K, Cd, ldc, items_per_part, min_parts, fixup,
                               ws, online, stream)))
         return st;
-    MPS_CUDA(cudaMemcpyAsync(C_host, Cd, (size_t)A->m * (size_t)ldc * 4, cudaMemcpyDeviceToHost,
-                             s), "D2H C");
+    MPS_CUDA(copy_rows(C_host, Cd, (size_t)ldc * 4, (size_t)K * 4, (size_t)A->m,
+                       cudaMemcpyDeviceToHost, s), "D2H C");
     return MPS_OK;
 }
 
@@ -1361,11 +1404,14 @@ static mps_status shard_impl(const CSR *A, const void *B, int32_t b_dtype, int64
     const size_t yb = align_up((size_t)(P + 1) * sizeof(IT), 256);
     int32_t *cx = (int32_t *)workspace;
     IT *cy = (IT *)((char *)workspace + xb);
-    void *rec = (char *)workspace + xb + yb;
+    unsigned *claims = (unsigned *)((char *)workspace + xb + yb);
+    void *rec = (char *)workspace + xb + yb + claim_bytes(K);
+    const int32_t nz = zeroable_claims(K, v);
     const int32_t trow = tail_rows[rank];
     MPS_CUDA(mps::launch_partition<IT>(A->row_ptr, A->m, A->nnz, D0, span, P, L, cx, cy,
                                        fix == mps::FIX_ATOMIC ? C_local : nullptr, ldc, X[rank],
-                                       K, trow, fix == mps::FIX_ATOMIC ? tail_out : nullptr, s),
+                                       K, trow, fix == mps::FIX_ATOMIC ? tail_out : nullptr,
+                                       claims, nz, s),
              "partition kernel");
     mps::SegArgsT<IT> a{};
     a.rp = A->row_ptr;
@@ -1385,7 +1431,7 @@ static mps_status shard_impl(const CSR *A, const void *B, int32_t b_dtype, int64
     a.tail = tail_out;
     a.nnz_end = (int64_t)Y[rank + 1];
     a.mail = mail;
-    return run_segments(a, b_dtype, K, v, fix, rec, s);
+    return run_segments(a, b_dtype, K, v, fix, rec, claims, nz > 0, s);
 }
 
 extern "C" {

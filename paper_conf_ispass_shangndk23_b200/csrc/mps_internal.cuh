@@ -75,7 +75,8 @@ struct SegArgsT {
     int32_t relu;        // epilogue: 1 = C = max(C, 0) (complete rows at the store; cut rows
                          // by launch_relu_split after the atomics, or in the carry reduce)
     TailMail mail;       // a6 peer-memory tail exchange (mail.on == 0: none)
-    unsigned *claim;     // set by the launcher: dynamic segment claims {next, done} or NULL
+    unsigned *claim;     // dynamic segment claims: this column tile's counter in the caller's
+                         // workspace, zero when the kernel starts (NULL: static assignment)
     int32_t deep;        // 1: deep-gather instantiation (fp32, 64-column tile, DRAM-bound B)
 };
 using SegArgs = SegArgsT<int32_t>;
@@ -87,12 +88,13 @@ template <typename IT>
 cudaError_t launch_partition(const IT *rp, int64_t m, int64_t nnz, int64_t d0,
                              int64_t span, int64_t P, int64_t L, int32_t *cx, IT *cy,
                              float *zero_C, int64_t ldc, int64_t row_base, int32_t K,
-                             int32_t tail_row, float *tail, cudaStream_t s);
+                             int32_t tail_row, float *tail, unsigned *claims, int32_t nclaims,
+                             cudaStream_t s);
 template <typename IT>
 cudaError_t launch_zero_split(const IT *rp, int32_t m, const int32_t *cx,
                               const IT *cy, int64_t P, float *C, int64_t ldc,
                               int64_t row_base, int32_t K, int32_t tail_row, float *tail,
-                              cudaStream_t s);
+                              unsigned *claims, int32_t nclaims, cudaStream_t s);
 template <typename IT>
 cudaError_t launch_segments(const SegArgsT<IT> &a, int b_dtype, int W, int V, int NR, int fix,
                             cudaStream_t s);
@@ -126,6 +128,12 @@ cudaError_t launch_xw_bf16_bcast(const void *X, int64_t n, int64_t F, int64_t ld
                                  int32_t nd, int64_t row_offset, int64_t ldb, cudaStream_t s);
 
 int num_sms();
+
+// Dynamic segment claims pay off from ~4 segments per warp; the launcher uses them only
+// when the schedule has that many per resident warp and the caller passed a claim
+// counter.  Smallest P for which they can be chosen (every instantiation runs >= 2
+// CTAs of kBlock threads per SM):
+inline int64_t seg_dynamic_min_parts() { return (int64_t)4 * 2 * (kBlock / 32) * num_sms(); }
 
 // ---------------------------------------------------------------------------------
 // device helpers

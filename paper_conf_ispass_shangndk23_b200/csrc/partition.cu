@@ -46,8 +46,11 @@ __global__ void __launch_bounds__(kBlock)
 partition_kernel(const IT *__restrict__ rp, int64_t m, int64_t nnz, int64_t d0,
                  int64_t span, int64_t P, int64_t L, int32_t *__restrict__ cx,
                  IT *__restrict__ cy, float *zero_C, int64_t ldc, int64_t row_base,
-                 int32_t K, int32_t tail_row, float *tail) {
+                 int32_t K, int32_t tail_row, float *tail, unsigned *claims, int32_t nclaims) {
     __shared__ IT s_rp[kPartWin];
+    // the segment kernel that follows on the stream claims segments from these counters
+    // (caller workspace); they start at zero
+    if (blockIdx.x == 0 && (int)threadIdx.x < nclaims) claims[threadIdx.x] = 0u;
     __shared__ int64_t s_x[2];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t pb = (int64_t)blockIdx.x * blockDim.x;
@@ -105,12 +108,14 @@ template <typename IT>
 cudaError_t launch_partition(const IT *rp, int64_t m, int64_t nnz, int64_t d0,
                              int64_t span, int64_t P, int64_t L, int32_t *cx, IT *cy,
                              float *zero_C, int64_t ldc, int64_t row_base, int32_t K,
-                             int32_t tail_row, float *tail, cudaStream_t s) {
+                             int32_t tail_row, float *tail, unsigned *claims,
+                             int32_t nclaims, cudaStream_t s) {
     const int64_t n = P + 1;
     const int64_t blocks = (n + kBlock - 1) / kBlock;
+    if (nclaims > kBlock) return cudaErrorInvalidValue;
     partition_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(rp, m, nnz, d0, span, P, L, cx, cy,
                                                          zero_C, ldc, row_base, K, tail_row,
-                                                         tail);
+                                                         tail, claims, claims ? nclaims : 0);
     return cudaGetLastError();
 }
 
@@ -120,7 +125,9 @@ template <typename IT>
 __global__ void __launch_bounds__(kBlock)
 zero_split_kernel(const IT *__restrict__ rp, int32_t m, const int32_t *__restrict__ cx,
                   const IT *__restrict__ cy, int64_t P, float *C, int64_t ldc,
-                  int64_t row_base, int32_t K, int32_t tail_row, float *tail) {
+                  int64_t row_base, int32_t K, int32_t tail_row, float *tail,
+                  unsigned *claims, int32_t nclaims) {
+    if (blockIdx.x == 0 && (int)threadIdx.x < nclaims) claims[threadIdx.x] = 0u;  // see above
     const int64_t p = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (p > P) return;
@@ -137,11 +144,13 @@ template <typename IT>
 cudaError_t launch_zero_split(const IT *rp, int32_t m, const int32_t *cx,
                               const IT *cy, int64_t P, float *C, int64_t ldc,
                               int64_t row_base, int32_t K, int32_t tail_row, float *tail,
-                              cudaStream_t s) {
+                              unsigned *claims, int32_t nclaims, cudaStream_t s) {
     const int64_t threads = (P + 1) * 32;
     const int64_t blocks = (threads + kBlock - 1) / kBlock;
+    if (nclaims > kBlock) return cudaErrorInvalidValue;
     zero_split_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(rp, m, cx, cy, P, C, ldc, row_base,
-                                                          K, tail_row, tail);
+                                                          K, tail_row, tail, claims,
+                                                          claims ? nclaims : 0);
     return cudaGetLastError();
 }
 
@@ -223,10 +232,11 @@ cudaError_t launch_validate(const IT *rp, const int32_t *col, int64_t m, int64_t
     template cudaError_t launch_partition<IT>(const IT *, int64_t, int64_t, int64_t, int64_t,  \
                                               int64_t, int64_t, int32_t *, IT *, float *,      \
                                               int64_t, int64_t, int32_t, int32_t, float *,     \
-                                              cudaStream_t);                                   \
+                                              unsigned *, int32_t, cudaStream_t);              \
     template cudaError_t launch_zero_split<IT>(const IT *, int32_t, const int32_t *,           \
                                                const IT *, int64_t, float *, int64_t, int64_t, \
-                                               int32_t, int32_t, float *, cudaStream_t);       \
+                                               int32_t, int32_t, float *, unsigned *, int32_t, \
+                                               cudaStream_t);                                  \
     template cudaError_t launch_write_stats<IT>(const IT *, int32_t, const int32_t *,          \
                                                 const IT *, int64_t, int64_t *, cudaStream_t); \
     template cudaError_t launch_validate<IT>(const IT *, const int32_t *, int64_t, int64_t,    \

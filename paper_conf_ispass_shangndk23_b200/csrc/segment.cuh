@@ -123,7 +123,11 @@ segment_kernel(const SegArgsT<IT> a) {
     asm volatile("griddepcontrol.wait;" ::: "memory");
 
     const uint64_t pol_last = a.l2_hints ? policy_evict_last() : policy_evict_normal();
-    const uint64_t pol_first = a.l2_hints ? policy_evict_first() : policy_evict_normal();
+    // col/val (and tail B rows with a hot bitmap) stream: evict_first, rebuilt at each use
+    // (one createpolicy) rather than held in two registers across the kernel
+    auto pol_first = [&]() -> uint64_t {
+        return a.l2_hints ? policy_evict_first() : policy_evict_normal();
+    };
     // segment indices are 32-bit (the launcher rejects P >= 2^31 - 2^20)
     const int wid = (int)blockIdx.x * kWarps + warp;
     const int wstride = (int)gridDim.x * kWarps;
@@ -218,8 +222,9 @@ segment_kernel(const SegArgsT<IT> a) {
                 fence_proxy_async_smem();
                 mbar_arrive_expect_tx(&bars[warp][pbuf], 2u * bytes);
                 if (bytes) {
-                    tma_load_1d(dc, col + cb, bytes, &bars[warp][pbuf], pol_first);
-                    tma_load_1d(dv, val + cb, bytes, &bars[warp][pbuf], pol_first);
+                    const uint64_t pf = pol_first();
+                    tma_load_1d(dc, col + cb, bytes, &bars[warp][pbuf], pf);
+                    tma_load_1d(dv, val + cb, bytes, &bars[warp][pbuf], pf);
                 }
             }
             const int rem = (int)(hi - (IT)ce);   // < 4 entries at the very end of the array
@@ -425,9 +430,10 @@ segment_kernel(const SegArgsT<IT> a) {
                     uint32_t hw[UL];
 #pragma unroll
                     for (int i = 0; i < UL; ++i) hw[i] = __ldg(hot + (cid[i] >> 5));
+                    const uint64_t pf = pol_first();
 #pragma unroll
                     for (int i = 0; i < UL; ++i) {
-                        const uint64_t pol = ((hw[i] >> (cid[i] & 31u)) & 1u) ? pol_last : pol_first;
+                        const uint64_t pol = ((hw[i] >> (cid[i] & 31u)) & 1u) ? pol_last : pf;
 #pragma unroll
                         for (int s = 0; s < V; ++s)
                             bv[i][s] = BV::load(reinterpret_cast<const TB *>(
@@ -487,38 +493,7 @@ segment_kernel(const SegArgsT<IT> a) {
                 write_row(a.rec + ((int64_t)seg * 2 + (single ? 0 : 1)) * a.kpad, false);
         }
     }
-    if constexpr (DYN) {                  // the last CTA resets the counter for reuse
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            __threadfence();
-            if (atomicAdd(a.claim + 1, 1u) == gridDim.x - 1) {
-                a.claim[0] = 0u;
-                a.claim[1] = 0u;
-                __threadfence();
-            }
-        }
-    }
     if (a.mail.on) tail_mail_epilogue(a.mail);   // a6 tail exchange (last CTA, last tile)
-}
-
-// Dynamic segment claims: self-resetting counter pairs {next, CTAs done}, zero at module
-// load; every launch takes the next slot (round robin over the whole library), so
-// launches in flight at the same time never share one.  One array per translation unit
-// (no relocatable device code); the slot index is global.
-constexpr int kClaimSlots = 1024;
-static __device__ unsigned g_claim[2 * kClaimSlots];
-inline std::atomic<uint32_t> g_claim_next{0};
-
-static unsigned *claim_slots() {
-    static unsigned *cache[64] = {nullptr};
-    int dev = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
-    if (!cache[dev]) {
-        void *p = nullptr;
-        if (cudaGetSymbolAddress(&p, g_claim) != cudaSuccess) return nullptr;
-        cache[dev] = (unsigned *)p;
-    }
-    return cache[dev];
 }
 
 // MPS_DYN (read per call): 0 = static segment assignment (warp w: w, w + warps, ...)
@@ -527,56 +502,65 @@ static bool dynamic_claims() {
     return e ? atoi(e) != 0 : true;
 }
 
+// Occupancy of one instantiation, per device (the carveout hint is a per-device
+// function attribute).  Idempotent, so concurrent first calls from several host
+// threads only repeat the same query.
+template <typename KFn>
+static cudaError_t seg_blocks_per_sm(KFn kstatic, KFn kdyn, int *out) {
+    static std::atomic<int> cache[64];
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev >= 0 && dev < 64) {
+        const int c = cache[dev].load(std::memory_order_relaxed);
+        if (c > 0) { *out = c; return cudaSuccess; }
+    }
+    // the staging buffers need the large shared-memory carveout for
+    // seg_min_blocks() CTAs per SM; MPS_CARVEOUT: carveout hint in percent (-1: none)
+    static const int carve = [] {
+        const char *ev = getenv("MPS_CARVEOUT");
+        return ev ? atoi(ev) : -1;
+    }();
+    if (carve >= 0) {
+        e = cudaFuncSetAttribute(kstatic, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(kdyn, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+        if (e != cudaSuccess) return e;
+    }
+    int bps = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kstatic, kBlock, 0);
+    if (e != cudaSuccess) return e;
+    if (bps < 1) bps = 1;
+    if (dev >= 0 && dev < 64) cache[dev].store(bps, std::memory_order_relaxed);
+    *out = bps;
+    return cudaSuccess;
+}
+
 template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false>
 static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
-    static int blocks_per_sm = 0;
-    if (blocks_per_sm == 0) {
-        // the staging buffers need the large shared-memory carveout for
-        // seg_min_blocks() CTAs per SM; without the hint the driver may pick a smaller one
-        // MPS_CARVEOUT: shared-memory carveout hint in percent (-1: none)
-        static const int carve = [] {
-            const char *e = getenv("MPS_CARVEOUT");
-            return e ? atoi(e) : -1;
-        }();
-        cudaError_t e = cudaSuccess;
-        if (carve >= 0) {
-            e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>,
-                                     cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-            if (e == cudaSuccess)
-                e = cudaFuncSetAttribute(segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>,
-                                         cudaFuncAttributePreferredSharedMemoryCarveout, carve);
-            if (e != cudaSuccess) return e;
-        }
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &blocks_per_sm, segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>, kBlock, 0);
-        if (e != cudaSuccess) return e;
-        if (blocks_per_sm < 1) blocks_per_sm = 1;
-    }
+    auto kst = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>;
+    auto kdy = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>;
+    int blocks_per_sm = 0;
+    cudaError_t e = seg_blocks_per_sm(kst, kdy, &blocks_per_sm);
+    if (e != cudaSuccess) return e;
     const int64_t warps_per_block = kBlock / 32;
     int64_t need = (a.P + warps_per_block - 1) / warps_per_block;
     const int64_t cap = (int64_t)blocks_per_sm * num_sms();
     const int64_t grid = need < cap ? need : cap;
     if (grid <= 0) return cudaSuccess;
     if (a.P >= (int64_t)0x7ff00000) return cudaErrorInvalidValue;   // 32-bit segment ids
-    SegArgsT<IT> arg = a;
-    arg.claim = nullptr;
-    bool dyn = false;
     // dynamic claims pay off from ~4 segments per warp (BASELINE graphs: 10-70 per warp,
     // 1-6% faster); at 1-3 per warp the opening burst of claims on one counter costs more
-    // than the balance gains (Table-II graphs, profiles/r01/dynamic_claims/)
-    if (a.P >= 4 * grid * warps_per_block && dynamic_claims()) {
-        unsigned *base = claim_slots();
-        if (base == nullptr) return cudaErrorInvalidSymbol;
-        arg.claim = base + 2 * (g_claim_next.fetch_add(1u) % kClaimSlots);
-        dyn = true;
-    }
+    // than the balance gains (Table-II graphs, profiles/r01/dynamic_claims/).  The counter
+    // (a.claim) lives in the caller's workspace and is zero when the kernel starts.
+    const bool dyn = a.claim != nullptr && a.P >= 4 * grid * warps_per_block && dynamic_claims();
     // launched with programmatic stream serialization (PDL): the CTAs may be scheduled
     // as the previous kernel's CTAs retire, hiding the launch gap (tens of percent of a
     // small graph's step); griddepcontrol.wait in the kernel keeps the data dependency.
     // MPS_PDL=0 launches plainly.
     static const int pdl = [] {
-        const char *e = getenv("MPS_PDL");
-        return e ? atoi(e) : 1;
+        const char *ev = getenv("MPS_PDL");
+        return ev ? atoi(ev) : 1;
     }();
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
@@ -588,9 +572,8 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = pdl ? 1 : 0;
-    if (dyn)
-        return cudaLaunchKernelEx(&cfg, segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>, arg);
-    return cudaLaunchKernelEx(&cfg, segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>, arg);
+    if (dyn) return cudaLaunchKernelEx(&cfg, kdy, a);
+    return cudaLaunchKernelEx(&cfg, kst, a);
 }
 
 // (W, V, NR) dispatch.  NR > 1 only with V == 1.

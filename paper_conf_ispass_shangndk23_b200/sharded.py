@@ -76,21 +76,46 @@ def replicate_B(B_rows: torch.Tensor, n: int, world: int, group=None) -> torch.T
     return full[:n]
 
 
+def _agree(ok: bool, device, group=None) -> bool:
+    """One all_reduce(MIN) of a success flag: True only if every rank succeeded."""
+    dev = device if dist.get_backend(group) == "nccl" else "cpu"
+    t = torch.tensor([1 if ok else 0], dtype=torch.int32, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+    return bool(int(t[0]) == 1)
+
+
 def _open_peers(buf: torch.Tensor, rank: int, world: int, group=None):
     """All ranks' device pointers to their `buf` (CUDA IPC), indexed by rank, plus the
-    bases this process opened (to close later)."""
+    bases this process opened (to close later).  Collective-safe: every rank takes part
+    in the same collectives whatever fails locally, and the ranks agree on success
+    before returning, so the call returns on all ranks or raises on all ranks."""
+    err = None
+    try:
+        mine = ipc_handle(buf)
+    except Exception as e:
+        mine, err = None, e
     allh = [None] * world
-    dist.all_gather_object(allh, ipc_handle(buf), group=group)
+    dist.all_gather_object(allh, mine, group=group)
     ptrs, opened = [], []
-    for g in range(world):
-        if g == rank:
-            ptrs.append(buf.data_ptr())
-            continue
-        h, off = allh[g]
-        base = ctypes.c_void_p()
-        L.mps_ipc_open_handle(ctypes.create_string_buffer(h, len(h)), ctypes.byref(base))
-        opened.append(base.value)
-        ptrs.append(base.value + off)
+    if err is None and all(h is not None for h in allh):
+        try:
+            for g in range(world):
+                if g == rank:
+                    ptrs.append(buf.data_ptr())
+                    continue
+                h, off = allh[g]
+                base = ctypes.c_void_p()
+                L.mps_ipc_open_handle(ctypes.create_string_buffer(h, len(h)), ctypes.byref(base))
+                opened.append(base.value)
+                ptrs.append(base.value + off)
+        except Exception as e:
+            err = e
+    else:
+        err = err or RuntimeError("a peer could not export its IPC handle")
+    if not _agree(err is None, buf.device, group):
+        for b in opened:
+            L.mps_ipc_close_handle(ctypes.c_void_p(b))
+        raise RuntimeError("peer mapping failed on some rank (this rank: %s)" % (err,))
     return ptrs, opened
 
 
@@ -152,12 +177,20 @@ class ShardedSpMM:
             ctypes.byref(self.a), K, dt, _p(self.X), rank, world, items_per_part, min_parts,
             _fix(fixup), ctypes.byref(nb))
         self.ws = _ws(nb.value, self.device)
-        self.tails = tails
+        self.tails = "nccl"
         self.epoch = 0
         self.mail = None
-        if tails == "p2p" and world > 1:
-            self.mail = Mailboxes(K, rank, world, self.device, group, ptrs=mailbox_ptrs)
-            self._mp = (ctypes.c_void_p * world)(*self.mail.ptrs)
+        if tails == "p2p":
+            self.enable_p2p(mailbox_ptrs)
+
+    def enable_p2p(self, mailbox_ptrs=None):
+        """Switch the tail exchange to peer memory: map every rank's mailbox (CUDA IPC;
+        collective over the group, succeeds or raises on every rank together)."""
+        self.tails = "p2p"
+        if self.world > 1 and self.mail is None:
+            self.mail = Mailboxes(self.K, self.rank, self.world, self.device, self.group,
+                                  ptrs=mailbox_ptrs)
+            self._mp = (ctypes.c_void_p * self.world)(*self.mail.ptrs)
 
     def local_p2p(self, B: torch.Tensor, stream=None, c0: int = 0, kt: int | None = None):
         """One step with the peer-memory tail exchange: afterwards this rank's C rows are
@@ -297,6 +330,8 @@ class ShardedGCNLayer:
     one process, dict(replicas=[ptr per rank], signals=[ptr per rank],
     mailboxes=[ptr per rank]); otherwise CUDA IPC over the process group."""
 
+    CONSUMED = 32     # first signal slot of the consumed-acks
+
     def __init__(self, row_ptr, col_idx, val, n, F, N, rank, world, device, tile_cols=64,
                  fixup="atomic", items_per_part=0, min_parts=0, group=None, peers=None):
         assert N % 16 == 0 and tile_cols % 16 == 0
@@ -304,7 +339,9 @@ class ShardedGCNLayer:
         self.device = torch.device(device)
         self.tile = min(tile_cols, N)
         self.tiles = [(c, min(self.tile, N - c)) for c in range(0, N, self.tile)]
-        assert len(self.tiles) <= 64
+        # signal slots: [0, 32) tile t produced (replicated) for an epoch, [32, 64) tile t
+        # consumed (this epoch's SpMM of tile t finished reading every replica)
+        assert len(self.tiles) <= self.CONSUMED
         self.sh = ShardedSpMM(row_ptr, col_idx, val, n, N, rank, world, device,
                               b_dtype=torch.bfloat16, fixup=fixup, items_per_part=items_per_part,
                               min_parts=min_parts, group=group, tails="p2p",
@@ -331,10 +368,16 @@ class ShardedGCNLayer:
         self.r0, self.r1 = int(self.sh.X[rank]), int(self.sh.X[rank + 1])
 
     def replicate(self, X_rows: torch.Tensor, Wt: torch.Tensor, stream):
-        """Enqueue B = X*W tile by tile into every replica, each tile followed by a signal."""
+        """Enqueue B = X*W tile by tile into every replica, each tile followed by a signal.
+        Tile t of this epoch overwrites every rank's replica only after every rank has
+        acknowledged that its SpMM of tile t of the previous epoch is done (consumed-ack
+        slot 32 + t), so back-to-back calls never overwrite B under a peer's gathers."""
         self.epoch += 1
         s = _stream(stream)
         for slot, (c0, kt) in enumerate(self.tiles):
+            if self.epoch > 1:
+                L.mps_peer_wait(ctypes.c_void_p(self._mysig), self.world, self.CONSUMED + slot,
+                                self.epoch - 1, s)
             dst = (ctypes.c_void_p * self.world)(*[p + 2 * c0 for p in self._dst])
             Wc = Wt[c0:c0 + kt]
             L.mps_xw_bf16_bcast(_p(X_rows), self.r1 - self.r0, X_rows.shape[1], X_rows.stride(0),
@@ -346,7 +389,11 @@ class ShardedGCNLayer:
         c0, kt = self.tiles[slot]
         L.mps_peer_wait(ctypes.c_void_p(self._mysig), self.world, slot, self.epoch,
                         _stream(stream))
-        return self.sh.local_p2p(self.B, stream=stream, c0=c0, kt=kt)
+        out = self.sh.local_p2p(self.B, stream=stream, c0=c0, kt=kt)
+        # consumed-ack: this rank no longer reads tile `slot` of its replica this epoch
+        L.mps_peer_signal(self._sig, self.world, self.rank, self.CONSUMED + slot, self.epoch,
+                          _stream(stream))
+        return out
 
     def __call__(self, X_rows: torch.Tensor, Wt: torch.Tensor, s_xw=None, s_agg=None):
         s_xw = s_xw or torch.cuda.Stream(self.device)

@@ -34,7 +34,7 @@ def test_header_symbols_exported():
 
 
 def test_abi_version_and_status_strings():
-    assert M.mps_abi_version() == 1
+    assert M.mps_abi_version() == 2
     assert M.mps_status_string(0) == b"MPS_OK"
     assert M.mps_status_string(4) == b"MPS_ERR_WORKSPACE"
 

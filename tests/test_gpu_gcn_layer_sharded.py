@@ -117,6 +117,67 @@ def test_sharded_gcn_layer_two_processes_ipc(tmp_path):
     assert sorted(int(k) for k, _ in oks) == [0, 1] and all(v == "true" for _, v in oks), r.stdout
 
 
+_WORKER_B2B = r'''
+import os, sys, json
+sys.path.insert(0, sys.argv[1])
+import numpy as np, torch, torch.distributed as dist
+import graphgen as G, oracle as O
+import paper_conf_ispass_shangndk23_b200 as M
+rank, world = int(os.environ["RANK"]), int(os.environ["WORLD_SIZE"])
+torch.cuda.set_device(0)
+dist.init_process_group("gloo")
+n, F, N = 1500, 64, 128
+rs = np.random.RandomState(3)
+rl = rs.randint(0, 10, size=n).astype(np.int32); rl[700] = 3000
+g = G.random_csr(n, n, rl, 4)
+W = torch.randint(-1, 2, (F, N), generator=torch.Generator().manual_seed(5)).to(torch.bfloat16)
+Xs = [torch.randint(-1, 2, (n, F), generator=torch.Generator().manual_seed(10 + k)).to(torch.bfloat16)
+      for k in range(5)]
+layer = M.ShardedGCNLayer(g.row_ptr, g.col_idx, g.val, n, F, N, rank, world, "cuda:0",
+                          tile_cols=32, items_per_part=31, min_parts=1)
+r0, r1 = layer.r0, layer.r1
+Wt = W.t().contiguous().cuda()
+Xd = [X.cuda()[r0:r1].contiguous() for X in Xs]
+s_xw, s_agg = torch.cuda.Stream(), torch.cuda.Stream()
+outs = []
+torch.cuda.synchronize(); dist.barrier()
+for k in range(5):          # back to back: no synchronisation, no barrier between calls
+    C = layer(Xd[k], Wt, s_xw=s_xw, s_agg=s_agg)
+    with torch.cuda.stream(s_agg):
+        outs.append(C.clone())
+torch.cuda.synchronize(); dist.barrier()
+ok = True
+x0, x1 = int(layer.sh.X[rank]), int(layer.sh.X[rank + 1])
+for k in range(5):
+    Bref = (Xs[k].double() @ W.double()).numpy()
+    ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bref, want_bound=False)
+    ok = ok and np.array_equal(outs[k].cpu().numpy().astype(np.float64), ref[x0:x1])
+layer.close()
+print(json.dumps({"rank": rank, "ok": bool(ok)}))
+dist.destroy_process_group()
+'''
+
+
+def test_sharded_gcn_layer_back_to_back_calls(tmp_path):
+    """ADVICE r1: a call must not overwrite a peer's B replica while that peer's SpMM of
+    the previous call still gathers from it (consumed-acks in ShardedGCNLayer).  Five
+    calls with a different X each, no synchronisation or barrier between them."""
+    import os, socket, subprocess, sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    w = tmp_path / "worker_b2b.py"
+    w.write_text(_WORKER_B2B)
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), str(w), root]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    oks = re.findall(r'\{"rank": (\d+), "ok": (true|false)\}', r.stdout)
+    assert sorted(int(k) for k, _ in oks) == [0, 1] and all(v == "true" for _, v in oks), r.stdout
+
+
 def _bf16_rne(a):
     """fp32 -> bf16 round-to-nearest-even (the kernels' __float2bfloat16_rn), as float64."""
     u = np.ascontiguousarray(a, np.float32).view(np.uint32).astype(np.uint64)

@@ -57,7 +57,52 @@ __global__ void __launch_bounds__(256) l2_stream(const uint4 *__restrict__ buf, 
     if (acc == 0x9e3779b9u) sink[0] = acc;
 }
 
-// mode 0: random row gathers (row_bytes in {16..512}); mode 1: streaming read.
+// Lean probes (modes 2 and 3): the index arithmetic above (two multiplicative hashes
+// and a runtime modulo per gather) costs more issue slots than the load itself, so
+// those probes are issue-bound below the L2 rate.  Here a power-of-two row count lets
+// one IMAD (LCG) + one shift pick a row, 16 gathers are in flight per lane, and the
+// streaming read issues 8 independent coalesced 512-B warp loads per iteration.
+template <int U>
+__global__ void __launch_bounds__(256) l2_gather_lean(const uint4 *__restrict__ tab,
+                                                      uint32_t shift, uint32_t row16,
+                                                      int iters, uint32_t *sink) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t grp = lane / row16, lr = lane % row16;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    uint32_t x = mix32(warp * 0x9E3779B9u + grp * 0x85ebca6bu + 7u);
+    uint32_t acc = 0;
+    for (int it = 0; it < iters; ++it) {
+        uint4 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            x = x * 1664525u + 1013904223u;
+            v[u] = ldg_na(tab + (uint64_t)(x >> shift) * row16 + lr);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) acc ^= v[u].x ^ v[u].y ^ v[u].z ^ v[u].w;
+    }
+    if (acc == 0x9e3779b9u) sink[0] = acc;
+}
+
+template <int U>
+__global__ void __launch_bounds__(256) l2_stream_lean(const uint4 *__restrict__ buf,
+                                                      uint32_t n16, int passes, uint32_t *sink) {
+    uint32_t acc = 0;
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    const uint32_t stride = gridDim.x * blockDim.x;
+    for (int p = 0; p < passes; ++p)
+        for (uint32_t i = tid; i + (U - 1) * stride < n16; i += U * stride) {
+            uint4 v[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) v[u] = ldg_na(buf + i + u * stride);
+#pragma unroll
+            for (int u = 0; u < U; ++u) acc ^= v[u].x ^ v[u].y ^ v[u].z ^ v[u].w;
+        }
+    if (acc == 0x9e3779b9u) sink[0] = acc;
+}
+
+// mode 0: random row gathers (row_bytes in {16..512}); mode 1: streaming read;
+// mode 2: lean random gathers (power-of-two rows); mode 3: lean streaming read.
 // Returns 0 on success; *gbs = best bytes read / time over the tried grid shapes.
 extern "C" int l2_probe_read_gbs2(int64_t bytes, int32_t row_bytes, int32_t mode, float *gbs,
                                   float *ms) {
@@ -77,12 +122,19 @@ extern "C" int l2_probe_read_gbs2(int64_t bytes, int32_t row_bytes, int32_t mode
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
     float best = 0.f, best_ms = 0.f;
-    const int per_sm[3] = {3, 4, 8};
-    for (int c = 0; c < 3; ++c) {
+    const int per_sm[4] = {3, 4, 6, 8};
+    uint32_t shift = 32;
+    uint32_t nrows2 = 1;
+    while (nrows2 * 2 <= nrows) { nrows2 *= 2; --shift; }
+    for (int c = 0; c < 4; ++c) {
         const int grid = sms * per_sm[c];
+        // lean stream: whole U*stride steps only (bytes counted exactly below)
+        const uint32_t st = (uint32_t)grid * 256u;
+        const uint32_t steps = (uint32_t)(n16 / (8ull * st));
         const int iters = 400;
         const int passes = 20;
         if (mode == 0) l2_gather<8><<<grid, 256>>>(buf, nrows, row16, 20, sink);
+        else if (mode == 2) l2_gather_lean<16><<<grid, 256>>>(buf, shift, row16, 10, sink);
         else l2_stream<<<grid, 256>>>(buf, n16, 1, sink);       // make it resident
         for (int rep = 0; rep < 3; ++rep) {
             cudaEventRecord(e0);
@@ -90,6 +142,13 @@ extern "C" int l2_probe_read_gbs2(int64_t bytes, int32_t row_bytes, int32_t mode
             if (mode == 0) {
                 l2_gather<8><<<grid, 256>>>(buf, nrows, row16, iters, sink);
                 moved = (double)grid * 256 * 16 * 8 * iters;   // 16 B per lane per gather
+            } else if (mode == 2) {
+                l2_gather_lean<16><<<grid, 256>>>(buf, shift, row16, iters / 2, sink);
+                moved = (double)grid * 256 * 16 * 16 * (iters / 2);
+            } else if (mode == 3) {
+                if (steps == 0) break;
+                l2_stream_lean<8><<<grid, 256>>>(buf, (uint32_t)(steps * 8ull * st), passes, sink);
+                moved = (double)steps * 8.0 * st * 16.0 * passes;
             } else {
                 l2_stream<<<grid, 256>>>(buf, n16, passes, sink);
                 moved = (double)n16 * 16 * passes;

@@ -20,8 +20,11 @@ P, Lp = M.plan(g.m, g.nnz, K, DT)
 cx = torch.empty(P + 1, dtype=torch.int32, device="cuda"); cy = torch.empty_like(cx)
 C = torch.empty(g.m, K, device="cuda")
 L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx), _p(cy), s)
+nb = ctypes.c_size_t()
+L.mps_spmm_workspace_bytes(ctypes.byref(a), K, DT, P, 1, ctypes.byref(nb))
+ws = torch.zeros(max(nb.value, 1), dtype=torch.uint8, device="cuda")
 def seg():
-    L.mps_spmm_segments(ctypes.byref(a), _p(B), DT, K, K, _p(C), K, _p(cx), _p(cy), P, 1, None, 0, s)
+    L.mps_spmm_segments(ctypes.byref(a), _p(B), DT, K, K, _p(C), K, _p(cx), _p(cy), P, 1, _p(ws), nb.value, s)
 def zero():
     L.mps_zero_split_rows(ctypes.byref(a), _p(cx), _p(cy), P, _p(C), K, K, s)
 def timeit(fn, pre=None, n=6):

@@ -1,6 +1,6 @@
 """NEXT-1: the paper's sensitivity study on B200 (sec. V, Figs. 5-7).
 
-For the 22 Table-II-shaped graphs (graphgen TABLE2) and K in {2, 4, 8, 16, 32, 64, 128}:
+For the 22 Table-II-shaped graphs (graphgen TABLE2) and K in {2, 4, 8, 16, 32, 64, 128, 256}:
   * merge-path cost sweep (items per warp segment; 0 = library default) -- Fig. 6;
   * at K=16 and the default cost: the Fig. 5 write statistic (#atomic row updates vs
     #regular row stores, mps_write_stats) and a parity check against the fp64 oracle.
@@ -19,7 +19,7 @@ import paper_conf_ispass_shangndk23_b200 as M
 from paper_conf_ispass_shangndk23_b200 import _lib as L
 from paper_conf_ispass_shangndk23_b200.api import _p, _stream
 
-KS = tuple(int(x) for x in os.environ.get("SENS_KS", "2 4 8 16 32 64 128").split())
+KS = tuple(int(x) for x in os.environ.get("SENS_KS", "2 4 8 16 32 64 128 256").split())
 DT = 1 if os.environ.get("SENS_DTYPE", "f32") == "bf16" else 0   # B dtype code
 COSTS = tuple(int(x) for x in os.environ.get("SENS_COSTS", "0 64 128 256 512 1024 2048 4096").split())
 
@@ -66,10 +66,13 @@ def main():
                 cx = torch.empty(P + 1, dtype=torch.int32, device="cuda")
                 cy = torch.empty_like(cx)
                 L.mps_partition(_p(A.row_ptr), g.m, g.nnz, 0, g.m + g.nnz, P, Lp, _p(cx), _p(cy), s)
+                nb = ctypes.c_size_t()
+                L.mps_spmm_workspace_bytes(ctypes.byref(a), K, DT, P, 1, ctypes.byref(nb))
+                ws = torch.zeros(max(nb.value, 1), dtype=torch.uint8, device="cuda")
 
                 def run():
                     L.mps_spmm(ctypes.byref(a), _p(B), DT, K, K, _p(C), K, _p(cx), _p(cy), P, 1,
-                               None, 0, _stream())
+                               _p(ws), nb.value, _stream())
                 ms = replay_ms(run)
                 row = {"graph": nm, "type": ty, "n": g.m, "nnz": g.nnz, "K": K, "cost": cost,
                        "P": P, "L": Lp, "ms": ms, "gflops": 2.0 * g.nnz * K / ms / 1e6}
