@@ -5,7 +5,7 @@ O=gpurun_out/${TAG:-r02b}
 mkdir -p $O
 python -c "import __graft_entry__ as e; e.build(); e.smoke()" > $O/smoke.txt 2>&1
 tail -2 $O/smoke.txt
-timeout 1800 python -m pytest tests -m gpu -q -p no:cacheprovider -x ${PYTEST_ARGS} > $O/tests_gpu.txt 2>&1
+timeout 1800 python -m pytest tests -m gpu -q -p no:cacheprovider ${PYTEST_ARGS} > $O/tests_gpu.txt 2>&1
 tail -5 $O/tests_gpu.txt
 timeout 600 python bench.py --out $O/bench_default.jsonl > $O/bench_default.log 2>&1; echo "bench rc=$?"
 tail -c 400 $O/bench_default.log
