@@ -52,7 +52,9 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--workload", default="reddit")
     ap.add_argument("--K", type=int, default=0)
-    ap.add_argument("--fixup", default="atomic")
+    ap.add_argument("--fixup", default="auto", choices=["auto", "atomic", "carry"],
+                    help="a4 fix-up: auto = the library's choice (carry on the small-graph "
+                         "fused path, atomic otherwise)")
     ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
     ap.add_argument("--items-per-part", type=int, default=0)
     ap.add_argument("--min-parts", type=int, default=0)
@@ -659,7 +661,7 @@ def main():
     traffic = None
     units = None
     prof = os.path.join(ROOT, "profiles", "traffic.json")
-    key = "%s-k%d-%s-%s" % (name, K, args.dtype, args.fixup)
+    key = "%s-k%d-%s-%s" % (name, K, args.dtype, "atomic" if args.fixup == "auto" else args.fixup)
     if os.path.exists(prof) and world == 1:
         with open(prof) as f:
             tj = json.load(f)
@@ -867,6 +869,9 @@ def main():
             "config": {
                 "workload": "%s-k%d" % (name, K), "graph": g.name, "n": g.m, "nnz": g.nnz,
                 "K": K, "b_dtype": args.dtype, "fixup": args.fixup,
+                "path": (("small_fused (1 kernel + carry reduction)"
+                          if online.path == L.MPS_PATH_SMALL_FUSED else
+                          "partition+segments") if world == 1 else "sharded"),
                 "num_parts": P, "items_per_part": Lp, "mode": "online (partition every step)",
                 "l2": {"write": "flushed before every timed step (2x L2 write, then 2x L2 read "
                                  "of a second buffer so no dirty lines remain; untimed)",

@@ -58,7 +58,8 @@ enum {
 
 /* How rows split across merge-path segments are settled (a4). */
 enum {
-    MPS_FIXUP_AUTO = 0,   /* library choice (currently ATOMIC)                        */
+    MPS_FIXUP_AUTO = 0,   /* library choice: CARRY on the small-graph fused path
+                           * (mps_spmm_online_path), ATOMIC otherwise                   */
     MPS_FIXUP_ATOMIC = 1, /* zero split rows, then one vector red.add per partial row  */
     MPS_FIXUP_CARRY = 2   /* partial rows to workspace, fixed-order reduction; deterministic */
 };
@@ -188,6 +189,23 @@ mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, 
                               int32_t K, float *C, int64_t ldc, int64_t items_per_part,
                               int64_t min_parts, int32_t fixup, int32_t epilogue,
                               void *workspace, size_t workspace_bytes, void *stream);
+
+/* Which kernels mps_spmm_online(_ex) launches for these arguments (same K, strides,
+ * pointers' alignment, items_per_part, min_parts and fixup as the call):
+ *  - MPS_PATH_PARTITION_SEGMENTS: the partition kernel (a2, plus the cut-row zeroing in
+ *    atomic mode), then the segment kernel per column tile (+ the carry reduction);
+ *  - MPS_PATH_SMALL_FUSED: small graphs -- row_ptr (m + 1 int32) and the segment staging
+ *    fit in one CTA's shared memory (<= 112 KB), L <= 512 items, one column tile
+ *    (K <= 32 x the lane vector width), int32 indices, fixup AUTO or CARRY: ONE kernel in
+ *    which every CTA stages the whole row_ptr and every warp computes its own segment's
+ *    coordinates (written to the workspace like the partition kernel's), walks it and
+ *    leaves the cut rows' pieces as carry records, then the carry reduction sums each cut
+ *    row in segment order (deterministic).  Both launches use programmatic dependent
+ *    launch.  MPS_SMALL=0 in the environment disables this path.                      */
+enum { MPS_PATH_PARTITION_SEGMENTS = 0, MPS_PATH_SMALL_FUSED = 1 };
+mps_status mps_spmm_online_path(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                int32_t K, const float *C, int64_t ldc, int64_t items_per_part,
+                                int64_t min_parts, int32_t fixup, int32_t *path_out);
 
 /* End-to-end call on HOST buffers: copies A and B host->device, runs the online path
  * and copies C device->host, all enqueued on `stream` (pinned host memory gives

@@ -15,6 +15,7 @@ MPS_OK, MPS_ERR_INVALID, MPS_ERR_UNSUPPORTED, MPS_ERR_CUDA, MPS_ERR_WORKSPACE, M
 MPS_FIXUP_AUTO, MPS_FIXUP_ATOMIC, MPS_FIXUP_CARRY = 0, 1, 2
 MPS_DT_F32, MPS_DT_BF16 = 0, 1
 MPS_EPI_NONE, MPS_EPI_RELU = 0, 1
+MPS_PATH_PARTITION_SEGMENTS, MPS_PATH_SMALL_FUSED = 0, 1
 
 _i64, _i32, _p, _sz = ctypes.c_int64, ctypes.c_int32, ctypes.c_void_p, ctypes.c_size_t
 
@@ -50,6 +51,7 @@ _SIGS = {
     "mps_spmm_workspace_bytes": [_p, _i32, _i32, _i64, _i32, _p],
     "mps_spmm": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _p, _sz, _p],
     "mps_spmm_ex": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _i32, _p, _p, _sz, _p],
+    "mps_spmm_online_path": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _p],
     "mps_spmm_online_ex": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _i32, _p, _sz,
                            _p],
     "mps_zero_split_rows": [_p, _p, _p, _i64, _p, _i64, _i32, _p],

@@ -324,37 +324,47 @@ def validate_csr(A: CSR, stream=None) -> int:
 
 
 class OnlineStep:
-    """One online MergePath-SpMM step as two library calls, for callers that time the
+    """One online MergePath-SpMM step as the library runs it, for callers that time the
     segment kernel on its own (bench.py's path of record; the full-size parity tests run
-    exactly this):
+    exactly this object).  Two forms, as ``mps_spmm_online_path`` decides:
 
-      a1 ``mps_plan`` (host, once) ->
-      a2 + a4 zeroing: ``mps_partition_split`` (atomic) / ``mps_partition`` (carry) ->
-      a3 (+ a4 carry reduction): ``mps_spmm_segments_hot`` (dynamic segment claims from
-      counters in ``ws``, programmatic dependent launch after the partition kernel).
+    * partition + segments (every graph that is not small):
+        a1 ``mps_plan`` (host, once) ->
+        a2 + a4 zeroing: ``mps_partition_split`` (atomic; ``mps_partition`` in carry
+        mode) ->
+        a3 (+ a4): ``mps_spmm_segments_hot`` (dynamic segment claims from counters in the
+        workspace, programmatic dependent launch behind the partition kernel);
+    * small-graph fused (``MPS_PATH_SMALL_FUSED``, fixup ``auto``/``carry``): one
+      ``mps_spmm_online_ex`` call -- one kernel computes the schedule and walks it, the
+      carry reduction settles the cut rows.
 
-    ``mps_spmm_online`` issues the same kernels in one call.  Buffers (coordinates, C,
-    workspace, optional hot-row bitmap) are allocated once and reused by every call, so
-    a call can be captured in a CUDA graph.  ``events``: (ev_after_partition,
-    ev_after_segments) recorded on the launching stream."""
+    ``mps_spmm_online`` issues the same kernels in one call.  Buffers (workspace with the
+    coordinates, C, optional hot-row bitmap) are allocated once and reused by every call,
+    so a call can be captured in a CUDA graph.  ``events``: (ev_after_partition,
+    ev_after_segments) recorded on the launching stream (the fused path records the first
+    one before its launch).  ``cx`` / ``cy``: the schedule's coordinates after a call."""
 
     def __init__(self, A: CSR, K: int, b_dtype=torch.float32, fixup="atomic",
                  items_per_part=0, min_parts=0, hot="auto", out: torch.Tensor | None = None):
         assert not A.wide, "OnlineStep: int32 indices (mps_csr)"
         self.A, self.K, self.fixup = A, K, _fix(fixup)
+        self.ipp, self.minp = items_per_part, min_parts
         self.dt = L.MPS_DT_BF16 if b_dtype == torch.bfloat16 else L.MPS_DT_F32
         self.a = A.struct()
         self.P, self.L = plan(A.m, A.nnz, K, self.dt, items_per_part, min_parts)
         dev = A.device
-        self.cx = torch.empty(self.P + 1, dtype=torch.int32, device=dev)
-        self.cy = torch.empty(self.P + 1, dtype=torch.int32, device=dev)
         self.C = torch.empty((A.m, K), dtype=torch.float32, device=dev) if out is None else out
         assert self.C.stride(1) == 1 and self.C.shape == (A.m, K)
+        # the online workspace: [coord_x][coord_y][claim counters][carry records][...]
         nb = ctypes.c_size_t()
-        L.mps_spmm_workspace_bytes(ctypes.byref(self.a), K, self.dt, self.P, self.fixup,
-                                   ctypes.byref(nb))
+        L.mps_spmm_online_workspace_bytes(ctypes.byref(self.a), K, self.dt, items_per_part,
+                                          min_parts, self.fixup, ctypes.byref(nb))
         self.ws_bytes = nb.value
         self.ws = _ws(nb.value, dev)
+        xb = -(-(self.P + 1) * 4 // 256) * 256
+        self.cx = self.ws[: (self.P + 1) * 4].view(torch.int32)
+        self.cy = self.ws[xb: xb + (self.P + 1) * 4].view(torch.int32)
+        self._seg_ofs = 2 * xb                     # mps_spmm_segments' workspace
         hr = ctypes.c_int64(-1)
         if hot == "auto":
             L.mps_hot_budget_rows(ctypes.byref(self.a), K, self.dt, ctypes.byref(hr))
@@ -366,12 +376,33 @@ class OnlineStep:
             self.hot_ws_bytes = nbh.value
             self.hot_ws = _ws(nbh.value, dev)
             self.hot_bm = torch.empty((A.n + 31) // 32, dtype=torch.int32, device=dev)
+        self.path = None
+
+    def resolve(self, B: torch.Tensor) -> int:
+        """The library's path for this B (MPS_PATH_*): depends on B's and C's alignment."""
+        path = ctypes.c_int32()
+        L.mps_spmm_online_path(ctypes.byref(self.a), _p(B), self.dt, B.stride(0), self.K,
+                               _p(self.C), self.C.stride(0), self.ipp, self.minp, self.fixup,
+                               ctypes.byref(path))
+        return path.value
 
     def __call__(self, B: torch.Tensor, events=None, stream=None):
         assert B.dim() == 2 and B.stride(1) == 1 and B.shape[1] == self.K
         assert _dtype_code(B) == self.dt
+        if self.path is None:
+            self.path = self.resolve(B)
         s = _stream(stream)           # looked up per call: CUDA-graph capture streams
+        st = stream or torch.cuda.current_stream(self.A.device)
         A, a = self.A, ctypes.byref(self.a)
+        if self.path == L.MPS_PATH_SMALL_FUSED:
+            if events is not None:
+                events[0].record(st)
+            L.mps_spmm_online_ex(a, _p(B), self.dt, B.stride(0), self.K, _p(self.C),
+                                 self.C.stride(0), self.ipp, self.minp, self.fixup,
+                                 L.MPS_EPI_NONE, _p(self.ws), self.ws_bytes, s)
+            if events is not None:
+                events[1].record(st)
+            return self.C
         if self.hot_bm is not None:   # hub rows of B -> L2 evict_last (recomputed per call)
             L.mps_hot_rows(a, self.hot_rows, _p(self.hot_bm), _p(self.hot_ws),
                            self.hot_ws_bytes, s)
@@ -381,18 +412,20 @@ class OnlineStep:
         else:
             L.mps_partition(_p(A.row_ptr), A.m, A.nnz, 0, A.m + A.nnz, self.P, self.L,
                             _p(self.cx), _p(self.cy), s)
-        st = stream or torch.cuda.current_stream(A.device)
         if events is not None:
             events[0].record(st)
+        seg_ws = self.ws[self._seg_ofs:]
         L.mps_spmm_segments_hot(a, _p(B), self.dt, B.stride(0), self.K, _p(self.C),
                                 self.C.stride(0), _p(self.cx), _p(self.cy), self.P, self.fixup,
-                                _p(self.hot_bm), _p(self.ws), self.ws_bytes, s)
+                                _p(self.hot_bm), _p(seg_ws), self.ws_bytes - self._seg_ofs, s)
         if events is not None:
             events[1].record(st)
         return self.C
 
     def launches(self, l2_bytes: int) -> int:
-        """Library kernels (and memsets) one call enqueues."""
+        """Library kernels one call launches (memsets not counted)."""
+        if self.path == L.MPS_PATH_SMALL_FUSED:
+            return 2
         eb = 2 if self.dt == L.MPS_DT_BF16 else 4
         tile = 512 if eb == 4 else 1024
         if self.A.n * self.K * eb > 0.5 * l2_bytes:

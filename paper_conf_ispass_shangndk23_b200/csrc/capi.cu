@@ -566,6 +566,30 @@ size_t online_bytes(int64_t P, int32_t K, const Vec &v, int fix, int64_t n = 0,
     return b;
 }
 
+// The one-launch small-graph path (small.cu): row_ptr and the col/val staging fit in one
+// CTA's shared memory, one column tile, int32 indices, no hot-row bitmap; chosen for
+// MPS_FIXUP_AUTO and MPS_FIXUP_CARRY (it settles cut rows with the carry records).
+// MPS_SMALL=0 disables it.
+bool small_possible(int64_t m, int64_t L) {
+    static const int on = [] {
+        const char *e = getenv("MPS_SMALL");
+        return e ? atoi(e) : 1;
+    }();
+    return on && L <= mps::kSmallMaxL && m + 1 < ((int64_t)1 << 30) &&
+           mps::small_smem_bytes(m, L) <= (size_t)mps::kSmallMaxSmem;
+}
+
+template <typename CSR>
+bool small_path_ok(const CSR *A, int32_t K, const Vec &v, int32_t fixup, int64_t L,
+                   int64_t hot_rows) {
+    if (sizeof(idx_t<CSR>) != 4 || fixup == MPS_FIXUP_ATOMIC || hot_rows >= 0) return false;
+    if (!small_possible(A->m, L) || A->nnz >= kMaxIndex) return false;
+    if (((uintptr_t)A->row_ptr) & 15u) return false;
+    int V, NR;
+    tile_geometry(K, v.W, &V, &NR);
+    return V == 1 && v.tile >= K;
+}
+
 template <typename CSR>
 mps_status online_ws_impl(const CSR *A, int32_t K, int32_t b_dtype, int64_t items_per_part,
                           int64_t min_parts, int32_t fixup, size_t *bytes) {
@@ -580,11 +604,88 @@ mps_status online_ws_impl(const CSR *A, int32_t K, int32_t b_dtype, int64_t item
     vmin.W = 1;
     vmin.tile = 128;
     const Vec v = choose_vec(K, b_dtype, nullptr, K ? K : 1, nullptr, K ? K : 1);
-    const int fix = resolve_fix(fixup);
+    // AUTO may take the small path, which needs the carry records
+    const int fix = (fixup == MPS_FIXUP_AUTO && sizeof(idx_t<CSR>) == 4 &&
+                     small_possible(A->m, L)) ? mps::FIX_CARRY : resolve_fix(fixup);
     const int64_t nh = hot_budget_rows(A->n, K, b_dtype) >= 0 ? A->n : 0;
     const size_t ys = sizeof(idx_t<CSR>);
     size_t a = online_bytes(P, K, v, fix, nh, ys), b = online_bytes(P, K, vmin, fix, nh, ys);
     *bytes = a > b ? a : b;
+    return MPS_OK;
+}
+
+template <typename CSR>
+mps_status small_online_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t ldb,
+                             int32_t K, float *C, int64_t ldc, int64_t P, int64_t L,
+                             const Vec &v, int32_t epilogue, void *workspace,
+                             size_t workspace_bytes, cudaStream_t s) {
+    const size_t need = online_bytes(P, K, v, mps::FIX_CARRY, 0, 4);
+    if (!workspace || workspace_bytes < need)
+        return fail(MPS_ERR_WORKSPACE, "workspace %zu < %zu", workspace_bytes, need);
+    const size_t xb = align_up((size_t)(P + 1) * 4, 256);
+    int32_t *cx = (int32_t *)workspace;
+    int32_t *cy = (int32_t *)((char *)workspace + xb);
+    float *rec = (float *)((char *)workspace + 2 * xb + claim_bytes(K));
+    int V, NR;
+    tile_geometry(K, v.W, &V, &NR);
+    static const int hints = [] {
+        const char *e = getenv("MPS_L2_HINTS");
+        return e ? atoi(e) : 1;
+    }();
+    mps::SmallArgs sa{};
+    sa.rp = (const int32_t *)A->row_ptr;
+    sa.col = A->col_idx;
+    sa.val = A->val;
+    sa.B = B;
+    sa.ldb = ldb;
+    sa.K = K;
+    sa.C = C;
+    sa.ldc = ldc;
+    sa.m = (int32_t)A->m;
+    sa.nnz = (int32_t)A->nnz;
+    sa.P = (int32_t)P;
+    sa.L = (int32_t)L;
+    sa.cx = cx;
+    sa.cy = cy;
+    sa.rec = rec;
+    sa.kpad = (int32_t)carry_kpad(K, v);
+    sa.relu = epilogue == MPS_EPI_RELU;
+    sa.l2_hints = hints;
+    MPS_CUDA(mps::launch_small_online(sa, b_dtype, v.W, NR, s), "small online kernel");
+    mps::SegArgsT<int32_t> a{};
+    a.rp = (const int32_t *)A->row_ptr;
+    a.C = C;
+    a.ldc = ldc;
+    a.K = K;
+    a.m = (int32_t)A->m;
+    a.cx = cx;
+    a.cy = cy;
+    a.P = P;
+    a.tail_row = -1;
+    a.rec = rec;
+    a.kpad = sa.kpad;
+    a.relu = sa.relu;
+    MPS_CUDA(mps::launch_carry_reduce(a, s), "carry reduce");
+    return MPS_OK;
+}
+
+// Which kernels the online call launches (mps_spmm_online_path).
+template <typename CSR>
+mps_status online_path_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t ldb,
+                            int32_t K, const float *C, int64_t ldc, int64_t items_per_part,
+                            int64_t min_parts, int32_t fixup, int32_t *path) {
+    mps_status st = check_csr(A, false);
+    if (st) return st;
+    if (!path) return fail(MPS_ERR_INVALID, "path_out NULL");
+    *path = MPS_PATH_PARTITION_SEGMENTS;
+    if (K <= 0 || A->m == 0) return MPS_OK;
+    int64_t P, L;
+    if ((st = plan_impl(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L,
+                        sizeof(idx_t<CSR>) == 8)))
+        return st;
+    const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n, A->m, A->nnz);
+    if (small_path_ok(A, K, v, fixup, L, hot_budget_rows(A->n, K, b_dtype)))
+        *path = MPS_PATH_SMALL_FUSED;
     return MPS_OK;
 }
 
@@ -604,9 +705,12 @@ mps_status online_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t 
     if ((st = plan_impl(A->m, A->nnz, K, b_dtype, items_per_part, min_parts, &P, &L,
                         sizeof(IT) == 8)))
         return st;
-    const int fix = resolve_fix(fixup);
     const Vec v = choose_vec(K, b_dtype, B, ldb, C, ldc, A->n, A->m, A->nnz);
     const int64_t hot_rows = hot_budget_rows(A->n, K, b_dtype);
+    if (small_path_ok(A, K, v, fixup, L, hot_rows))
+        return small_online_impl(A, B, b_dtype, ldb, K, C, ldc, P, L, v, epilogue, workspace,
+                                 workspace_bytes, (cudaStream_t)stream);
+    const int fix = resolve_fix(fixup);
     const int64_t nh = hot_rows >= 0 ? A->n : 0;
     const size_t need = online_bytes(P, K, v, fix, nh, sizeof(IT));
     if (!workspace || workspace_bytes < need)
@@ -770,6 +874,13 @@ mps_status mps_spmm_online(const mps_csr *A, const void *B, int32_t b_dtype, int
                            size_t workspace_bytes, void *stream) {
     return online_ex_impl(A, B, b_dtype, ldb, K, C, ldc, items_per_part, min_parts, fixup,
                           MPS_EPI_NONE, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_online_path(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                int32_t K, const float *C, int64_t ldc, int64_t items_per_part,
+                                int64_t min_parts, int32_t fixup, int32_t *path_out) {
+    return online_path_impl(A, B, b_dtype, ldb, K, C, ldc, items_per_part, min_parts, fixup,
+                            path_out);
 }
 
 mps_status mps_spmm_online_ex(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,

@@ -82,6 +82,31 @@ struct SegArgsT {
 using SegArgs = SegArgsT<int32_t>;
 using SegArgs64 = SegArgsT<int64_t>;
 
+// The one-launch online step for small graphs (small.cu): every CTA stages the whole
+// row_ptr in shared memory; each warp computes its segment's coordinates, walks it, and
+// leaves the cut rows' pieces in the carry records for carry_reduce_kernel.
+struct SmallArgs {
+    const int32_t *rp;
+    const int32_t *col;
+    const float *val;
+    const void *B;
+    int64_t ldb;
+    int32_t K;
+    float *C;
+    int64_t ldc;
+    int32_t m, nnz;
+    int32_t P, L;
+    int32_t *cx, *cy;   // out: coordinates of the P + 1 diagonals
+    float *rec;         // carry records [P][2][kpad]
+    int32_t kpad;
+    int32_t relu;
+    int32_t l2_hints;
+};
+constexpr int kSmallMaxSmem = 112 * 1024;   // row_ptr + col/val staging per CTA (2 CTAs/SM)
+constexpr int kSmallMaxL = 512;             // items per segment
+size_t small_smem_bytes(int64_t m, int64_t L);
+cudaError_t launch_small_online(const SmallArgs &a, int b_dtype, int W, int NR, cudaStream_t s);
+
 // Host launchers (defined in the .cu files).  IT = int32_t or int64_t (row_ptr and the
 // nnz coordinate y).
 template <typename IT>

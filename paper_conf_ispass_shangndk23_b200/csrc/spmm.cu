@@ -87,6 +87,9 @@ __device__ __forceinline__ void carry_one(const SegArgsT<IT> &a) {
 template <typename IT>
 __global__ void __launch_bounds__(kBlock)
 carry_reduce_kernel(const SegArgsT<IT> a) {
+    // launched with programmatic dependent launch behind the kernel that wrote the
+    // records: wait for it before reading them (a no-op without PDL)
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     carry_one(a);
     if (a.mail.on) tail_mail_epilogue(a.mail);   // a6 tail exchange (carry mode)
 }
@@ -95,8 +98,17 @@ template <typename IT>
 cudaError_t launch_carry_reduce(const SegArgsT<IT> &a, cudaStream_t s) {
     const int64_t threads = (a.P + 1) * 32;
     const int64_t blocks = (threads + kBlock - 1) / kBlock;
-    carry_reduce_kernel<IT><<<(unsigned)blocks, kBlock, 0, s>>>(a);
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3(kBlock);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, carry_reduce_kernel<IT>, a);
 }
 
 // Epilogue for the rows cut by a schedule boundary in atomic mode: they are final only
