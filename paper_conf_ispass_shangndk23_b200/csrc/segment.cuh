@@ -71,6 +71,11 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP_MINNR
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
+// slow path of the segment walk: 1 = step by step (one warp instruction's NR non-zeros at
+// a time), 0 = one pass over the whole batch per row touching it
+#ifndef MPS_SLOW_STEPS
+#define MPS_SLOW_STEPS 1
+#endif
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
 #endif
@@ -160,7 +165,10 @@ segment_kernel(const SegArgsT<IT> a) {
         return ys - (IT)(((uintptr_t)(col + ys) & 15u) >> 2);
     };
     // TMA may not read past the last 16-B boundary inside [.., nnz_end)
-    const int64_t lim4 = a.nnz_end - (int64_t)(((uintptr_t)(col + a.nnz_end) & 15u) >> 2);
+    // (recomputed where needed: a.nnz_end lives in the parameter bank, not a register)
+    auto lim4 = [&]() -> int64_t {
+        return a.nnz_end - (int64_t)(((uintptr_t)(col + a.nnz_end) & 15u) >> 2);
+    };
 
     // ---------------- this warp's sequence of segments ---------------------------------
     // static: wid, wid + wstride, ...; dynamic (a.claim != nullptr): each warp claims its
@@ -216,7 +224,8 @@ segment_kernel(const SegArgsT<IT> a) {
         float *dv = st.val[pbuf];
         if (!direct) {
             int64_t ce = cb + (((int64_t)hi - cb + 3) & ~3ll);
-            if (ce > lim4) ce = lim4 > cb ? lim4 : cb;
+            const int64_t l4 = lim4();
+            if (ce > l4) ce = l4 > cb ? l4 : cb;
             const uint32_t bytes = (uint32_t)(ce - cb) * 4u;
             if (lane == 0) {
                 fence_proxy_async_smem();
@@ -246,8 +255,8 @@ segment_kernel(const SegArgsT<IT> a) {
     prod_load_seg();
     produce();
 
-    uint32_t phase0 = 0, phase1 = 0;
-    int cbuf = 0;
+    // chunks consumed so far: buffer = bit 0, mbarrier phase of that buffer = bit 1
+    uint32_t ccount = 0;
 
     for (; cur < nseg; cur = nxt, nxt = cur < nseg ? claim_after(cur) : nseg) {
         const int seg = cur;
@@ -377,15 +386,14 @@ segment_kernel(const SegArgsT<IT> a) {
 
         for (int k = 0; k < nch; ++k) {
             if (!direct) {
-                mbar_wait(&bars[warp][cbuf], cbuf ? phase1 : phase0);
-                if (cbuf) phase1 ^= 1u; else phase0 ^= 1u;
+                mbar_wait(&bars[warp][ccount & 1u], (ccount >> 1) & 1u);
             }
             __syncwarp();
             produce();                  // next chunk into the other buffer
             if (direct) __syncwarp();
             const int cb = sb + k * kCH;
-            const int32_t *sc = st.col[cbuf];
-            const float *sv = st.val[cbuf];
+            const int32_t *sc = st.col[ccount & 1u];
+            const float *sv = st.val[ccount & 1u];
             int q = ys - cb;
             q = q > 0 ? (q / U) * U : 0;
             const int qend = min(kCH, ye - cb);
@@ -458,6 +466,40 @@ segment_kernel(const SegArgsT<IT> a) {
                     }
                 } else {
                     // slow path: the batch crosses row ends (or the segment's edges).
+#if MPS_SLOW_STEPS
+                    // Step by step (step i = the NR non-zeros j0 + i*NR .. + NR-1 of one
+                    // warp instruction): rows that end before the step are settled, then
+                    // a step inside row r is one predicated FMA; only a step that a row
+                    // end cuts takes one pass per row.  Cost ~ UL + (row ends) FMA
+                    // passes, not (1 + row ends) * UL as with whole-batch passes -- the
+                    // difference on short-row graphs (R-MAT: median row length 1).
+                    float vl[UL];
+#pragma unroll
+                    for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
+                    const int lo = j0 > ys ? j0 : ys;            // the batch's part of the
+                    const int hi = (j0 + U < ye) ? j0 + U : ye;  // segment: [lo, hi)
+#pragma unroll
+                    for (int i = 0; i < UL; ++i) {
+                        const int jb = j0 + i * NR;
+                        const int sb = jb > lo ? jb : lo;
+                        const int se = (jb + NR < hi) ? jb + NR : hi;
+                        if (sb < se) {                           // warp-uniform
+                            while (sb >= rend) finish_row();     // rows ending before the step
+                            const int j = jb + grp;
+                            if (se <= rend) {
+                                if (j >= sb && j < se) fma_row(vl[i], bv[i]);
+                            } else {                             // a row end inside the step
+                                int c = sb;
+                                while (c < se) {
+                                    while (c >= rend) finish_row();
+                                    const int lim = rend < se ? rend : se;
+                                    if (j >= c && j < lim) fma_row(vl[i], bv[i]);
+                                    c = lim;
+                                }
+                            }
+                        }
+                    }
+#else
                     // One pass per row intersecting the batch: predicated FMAs for the
                     // non-zeros of the current row, then settle the row.
                     float vl[UL];
@@ -475,9 +517,10 @@ segment_kernel(const SegArgsT<IT> a) {
                         }
                         jc = lim;
                     }
+#endif
                 }
             }
-            cbuf ^= 1;
+            ++ccount;
         }
         // rows whose end item lies in this segment after its last non-zero
         while (r < xe) finish_row();
