@@ -620,6 +620,10 @@ def main():
         evs[i][0].record(stream)
         run_step((evs[i][1], evs[i][2]))
         evs[i][3].record(stream)
+        # each step runs alone on the GPU (the protocol of the cuSPARSE reference point:
+        # flush, event, call, event, synchronise); for the tiny graphs the launch of a
+        # step queued behind the previous one otherwise adds several microseconds
+        torch.cuda.synchronize(dev)
     torch.cuda.synchronize(dev)
     barrier()
     wall = time.perf_counter() - wall0
@@ -873,6 +877,8 @@ def main():
                           if online.path == L.MPS_PATH_SMALL_FUSED else
                           "partition+segments") if world == 1 else "sharded"),
                 "num_parts": P, "items_per_part": Lp, "mode": "online (partition every step)",
+                "timing": "CUDA events around each step on the launching stream, every step "
+                          "synchronised (the cuSPARSE reference's protocol); value = mean",
                 "l2": {"write": "flushed before every timed step (2x L2 write, then 2x L2 read "
                                  "of a second buffer so no dirty lines remain; untimed)",
                        "read": "flushed before every timed step (2x L2 read, untimed)",
@@ -890,6 +896,7 @@ def main():
             "segment_ms_steps": [round(x, 4) for x in seg_ms],
             "step_ms_p10_p90": [float(np.percentile(step_ms, 10)),
                                 float(np.percentile(step_ms, 90))],
+            "step_ms_min_median": [float(np.min(step_ms)), float(np.median(step_ms))],
             "wall_s_timed_region": wall,
             "roofline": dict(roof, kernel="segment_kernel (a3)", traffic=traffic,
                              algorithmic_bytes_per_launch=int(seg_bytes), units=units),

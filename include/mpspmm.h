@@ -143,6 +143,22 @@ mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, i
                              const int32_t *coord_y, int64_t num_parts, int32_t fixup,
                              void *workspace, size_t workspace_bytes, void *stream);
 
+/* The Fig. 5 statistic counted where the segment kernel writes: mps_spmm
+ * (zeroing of the cut rows in atomic mode, then the segment kernel with its debug
+ * counters on) writing C as mps_spmm does, and counts (device int64[3], zeroed first):
+ *   [0] partial-row updates issued (Alg. 2 lines 5, 9, 13: red.add in atomic mode, a
+ *       carry record in carry mode),
+ *   [1] partial start pieces that are empty (the segment starts on a row's end item),
+ *       whose add the kernel elides -- Alg. 2 counts them as updates, so [0] + [1] is
+ *       the paper's #atomic,
+ *   [2] complete-row stores (Alg. 2 line 15), the paper's #regular.
+ * Column tile 0 is counted.  Same workspace as mps_spmm.                           */
+mps_status mps_spmm_write_counts(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                 int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                                 const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                                 int64_t *counts, void *workspace, size_t workspace_bytes,
+                                 void *stream);
+
 /* Degree-aware L2 residency (a B200 addition, not in the paper).  When B does not fit
  * in L2, the B rows gathered most often (hub columns of a power-law A) should stay in
  * L2 and the long tail should stream.  mps_hot_rows counts the non-zeros of every

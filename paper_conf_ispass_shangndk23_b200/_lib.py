@@ -51,6 +51,8 @@ _SIGS = {
     "mps_spmm_workspace_bytes": [_p, _i32, _i32, _i64, _i32, _p],
     "mps_spmm": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _p, _sz, _p],
     "mps_spmm_ex": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _i32, _p, _p, _sz, _p],
+    "mps_spmm_write_counts": [_p, _p, _i32, _i64, _i32, _p, _i64, _p, _p, _i64, _i32, _p, _p,
+                              _sz, _p],
     "mps_spmm_online_path": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _p],
     "mps_spmm_online_ex": [_p, _p, _i32, _i64, _i32, _p, _i64, _i64, _i64, _i32, _i32, _p, _sz,
                            _p],

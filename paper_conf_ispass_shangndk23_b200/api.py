@@ -435,3 +435,28 @@ class OnlineStep:
         if self.hot_bm is not None:
             n += 4
         return n
+
+
+def write_counts(A: CSR, B: torch.Tensor, schedule: Schedule, fixup="atomic",
+                 out: torch.Tensor | None = None, stream=None):
+    """Fig. 5 statistic as the segment kernel writes it (mps_spmm_write_counts): runs the
+    offline SpMM with the kernel's counters on.  Returns (C, (issued partial-row updates,
+    elided empty partial pieces, complete-row stores)); issued + elided is Alg. 2's
+    #atomic and the last one its #regular."""
+    K = B.shape[1]
+    dt = _dtype_code(B)
+    C = _keep(torch.empty((A.m, K), dtype=torch.float32, device=A.device), stream) \
+        if out is None else out
+    a = A.struct()
+    nb = ctypes.c_size_t()
+    L.mps_spmm_workspace_bytes(ctypes.byref(a), K, dt, schedule.num_parts, _fix(fixup),
+                               ctypes.byref(nb))
+    ws = _ws(nb.value, A.device, stream)
+    cnt = _keep(torch.empty(3, dtype=torch.int64, device=A.device), stream)
+    L.mps_spmm_write_counts(ctypes.byref(a), _p(B), dt, B.stride(0), K, _p(C), C.stride(0),
+                            _p(schedule.coord_x), _p(schedule.coord_y), schedule.num_parts,
+                            _fix(fixup), _p(cnt), _p(ws), nb.value, _stream(stream))
+    if stream is not None:
+        stream.synchronize()
+    c = cnt.cpu().tolist()
+    return C, (int(c[0]), int(c[1]), int(c[2]))

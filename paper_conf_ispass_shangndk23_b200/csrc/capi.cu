@@ -261,6 +261,7 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
         a.rec = (float *)workspace;
         a.kpad = (int32_t)carry_kpad(K, v);
         a.claim = claims ? claims + c0 / v.tile : nullptr;
+        if (c0 > 0) a.wstat = nullptr;      // the write statistic counts column tile 0
         // TMA staging needs col and val equally aligned modulo 16 B
         a.direct = ((((uintptr_t)base.col) ^ ((uintptr_t)base.val)) & 15u) != 0;
         static const int hints = [] {
@@ -453,7 +454,8 @@ mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t l
                          float *C, int64_t ldc, const int32_t *coord_x,
                          const idx_t<CSR> *coord_y, int64_t num_parts, int32_t fixup,
                          const uint32_t *hot_bitmap, int32_t relu, void *workspace,
-                         size_t workspace_bytes, void *stream, bool claims_zeroed = false) {
+                         size_t workspace_bytes, void *stream, bool claims_zeroed = false,
+                         unsigned long long *wstat = nullptr) {
     mps_status st = check_csr(A);
     if (st) return st;
     if ((st = check_dense(B, b_dtype, ldb, K, C, ldc, A))) return st;
@@ -484,6 +486,7 @@ mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t l
     a.nnz_end = A->nnz;
     a.hot = hot_bitmap;
     a.relu = relu;
+    a.wstat = wstat;
     return run_segments(a, b_dtype, K, v, fix, (char *)workspace + claim_bytes(K),
                         (unsigned *)workspace, claims_zeroed, (cudaStream_t)stream);
 }
@@ -820,6 +823,24 @@ mps_status mps_spmm_segments(const mps_csr *A, const void *B, int32_t b_dtype, i
                              void *workspace, size_t workspace_bytes, void *stream) {
     return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
                          nullptr, 0, workspace, workspace_bytes, stream);
+}
+
+mps_status mps_spmm_write_counts(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,
+                                 int32_t K, float *C, int64_t ldc, const int32_t *coord_x,
+                                 const int32_t *coord_y, int64_t num_parts, int32_t fixup,
+                                 int64_t *counts, void *workspace, size_t workspace_bytes,
+                                 void *stream) {
+    if (!counts) return fail(MPS_ERR_INVALID, "counts NULL");
+    cudaStream_t s = (cudaStream_t)stream;
+    MPS_CUDA(cudaMemsetAsync(counts, 0, 3 * sizeof(int64_t), s), "zero counts");
+    mps_status st = check_csr(A);
+    if (st) return st;
+    if (resolve_fix(fixup) == mps::FIX_ATOMIC && K > 0 && A->m > 0 &&
+        (st = zero_split_impl(A, coord_x, coord_y, num_parts, C, ldc, K, stream)))
+        return st;
+    return segments_impl(A, B, b_dtype, ldb, K, C, ldc, coord_x, coord_y, num_parts, fixup,
+                         nullptr, 0, workspace, workspace_bytes, stream, false,
+                         reinterpret_cast<unsigned long long *>(counts));
 }
 
 mps_status mps_spmm_segments_hot(const mps_csr *A, const void *B, int32_t b_dtype, int64_t ldb,

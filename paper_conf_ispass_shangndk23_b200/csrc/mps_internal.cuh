@@ -78,6 +78,10 @@ struct SegArgsT {
     unsigned *claim;     // dynamic segment claims: this column tile's counter in the caller's
                          // workspace, zero when the kernel starts (NULL: static assignment)
     int32_t deep;        // 1: deep-gather instantiation (fp32, 64-column tile, DRAM-bound B)
+    unsigned long long *wstat;  // Fig. 5 counters of what the kernel wrote (NULL: off):
+                                // [0] partial-row updates (atomic / carry record),
+                                // [1] empty partial start pieces whose add was elided,
+                                // [2] complete-row stores
 };
 using SegArgs = SegArgsT<int32_t>;
 using SegArgs64 = SegArgsT<int64_t>;
@@ -163,6 +167,11 @@ inline int64_t seg_dynamic_min_parts() { return (int64_t)4 * 2 * (kBlock / 32) *
 // ---------------------------------------------------------------------------------
 // device helpers
 // ---------------------------------------------------------------------------------
+// Fig. 5 write statistic counted where the kernel writes; off (NULL) on the
+// hot path, where it costs one uniform test per row end.
+__device__ __forceinline__ void count_write(unsigned long long *wstat, int lane, int k) {
+    if (wstat != nullptr && lane == 0) atomicAdd(wstat + k, 1ull);
+}
 __device__ __forceinline__ int ld_stream_i32(const int32_t *p) {
     int v;
     asm volatile("ld.global.cs.s32 %0, [%1];" : "=r"(v) : "l"(p));
@@ -338,6 +347,24 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
+// Ampere-style asynchronous copies global -> shared (LDGSTS): many in flight per thread
+// without a register round trip; cp_async_wait_all() then a barrier makes them visible.
+__device__ __forceinline__ void cp_async16(void *dst_smem, const void *src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(smem_u32(dst_smem)), "l"(src)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async4(void *dst_smem, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(smem_u32(dst_smem)), "l"(src)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async8(void *dst_smem, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" :: "r"(smem_u32(dst_smem)), "l"(src)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+    asm volatile("cp.async.wait_all;" ::: "memory");
+}
+
 // global -> shared bulk copy of `bytes` (multiple of 16, both addresses 16-B aligned),
 // completion counted on `bar`; L2 evict_first (streamed once).
 __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t bytes,

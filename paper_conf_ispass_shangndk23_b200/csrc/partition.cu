@@ -69,7 +69,13 @@ partition_kernel(const IT *__restrict__ rp, int64_t m, int64_t nnz, int64_t d0,
     const int64_t wn = xhi - xlo + 1;           // candidates x in [xlo, xhi]
     const bool staged = wn <= kPartWin;
     if (staged) {
-        for (int64_t i = threadIdx.x; i < wn; i += blockDim.x) s_rp[i] = __ldg(rp + xlo + i);
+        // asynchronous copies, all in flight at once: one memory round trip for the window
+        // (a load-then-store loop serialises one round trip per iteration)
+        for (int64_t i = threadIdx.x; i < wn; i += blockDim.x) {
+            if constexpr (sizeof(IT) == 8) cp_async8(s_rp + i, rp + xlo + i);
+            else cp_async4(s_rp + i, rp + xlo + i);
+        }
+        cp_async_wait_all();
         __syncthreads();
     }
     const int64_t p = pb + threadIdx.x;

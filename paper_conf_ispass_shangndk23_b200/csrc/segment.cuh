@@ -71,10 +71,12 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP_MINNR
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
-// slow path of the segment walk: 1 = step by step (one warp instruction's NR non-zeros at
-// a time), 0 = one pass over the whole batch per row touching it
+// slow path of the segment walk: 0 = one pass over the whole batch per row touching it;
+// 1 = step by step (one warp instruction's NR non-zeros at a time).  Measured on B200
+// (profiles/r02/slow_steps.md): the step form is 1.6x slower on R-MAT and 2.3x on
+// products (register spills and serialised per-step control flow), so 0 stays.
 #ifndef MPS_SLOW_STEPS
-#define MPS_SLOW_STEPS 1
+#define MPS_SLOW_STEPS 0
 #endif
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
@@ -340,20 +342,27 @@ segment_kernel(const SegArgsT<IT> a) {
 
         // Row r ends inside this segment: settle it and move to row r + 1.
         auto finish_row = [&]() {
-            combine();
+            // an empty row has nothing in any lane group: no butterfly (R-MAT: 48% empty)
+            if (rend != rbeg) combine();
             if (r == xs && start_in) {
                 // partial start row (Alg. 2 lines 8-9): atomic, or carry record slot 0
                 if (FIX == FIX_ATOMIC) {
-                    if (ys < rend)
+                    if (ys < rend) {
                         write_row((r == a.tail_row) ? a.tail
                                                     : a.C + ((int64_t)r - a.row_base) * a.ldc,
                                   true);
+                        count_write(a.wstat, lane, 0);
+                    } else {
+                        count_write(a.wstat, lane, 1);   // empty piece: the add is elided
+                    }
                 } else {
                     write_row(a.rec + ((int64_t)seg * 2) * a.kpad, false);
+                    count_write(a.wstat, lane, 0);
                 }
             } else {
                 // complete row (line 15): plain store, no initialisation of C needed
                 write_row(a.C + ((int64_t)r - a.row_base) * a.ldc, false, a.relu != 0);
+                count_write(a.wstat, lane, 2);
             }
 #pragma unroll
             for (int s = 0; s < V; ++s)
@@ -534,6 +543,7 @@ segment_kernel(const SegArgsT<IT> a) {
                           true);
             else
                 write_row(a.rec + ((int64_t)seg * 2 + (single ? 0 : 1)) * a.kpad, false);
+            count_write(a.wstat, lane, 0);
         }
     }
     if (a.mail.on) tail_mail_epilogue(a.mail);   // a6 tail exchange (last CTA, last tile)

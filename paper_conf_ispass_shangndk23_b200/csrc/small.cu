@@ -64,13 +64,15 @@ __global__ void __launch_bounds__(kBlock) small_online_kernel(const SmallArgs a)
     // the inputs may come from the previous kernel of the stream (PDL: launched early)
     asm volatile("griddepcontrol.wait;" ::: "memory");
 
-    // stage row_ptr[0..m]: one round of independent 16-B loads
+    // stage row_ptr[0..m]: asynchronous 16-B copies, all in flight at once (one memory
+    // round trip; a load-then-store loop would serialise one round trip per iteration)
     {
         const int n4 = (m + 1) >> 2;
         const int4 *src = reinterpret_cast<const int4 *>(a.rp);
         int4 *dst = reinterpret_cast<int4 *>(s_rp);
-        for (int i = threadIdx.x; i < n4; i += blockDim.x) dst[i] = __ldg(src + i);
-        for (int i = 4 * n4 + threadIdx.x; i <= m; i += blockDim.x) s_rp[i] = __ldg(a.rp + i);
+        for (int i = threadIdx.x; i < n4; i += blockDim.x) cp_async16(dst + i, src + i);
+        for (int i = 4 * n4 + threadIdx.x; i <= m; i += blockDim.x) cp_async4(s_rp + i, a.rp + i);
+        cp_async_wait_all();
     }
     __syncthreads();
     const int p = (int)blockIdx.x * kWarps + warp;
@@ -95,9 +97,10 @@ __global__ void __launch_bounds__(kBlock) small_online_kernel(const SmallArgs a)
     // col/val of the segment's non-zeros [ys, ye) (<= L entries)
     const int nn = ye - ys;
     for (int t = lane; t < nn; t += 32) {
-        s_col[t] = __ldg(a.col + ys + t);
-        s_val[t] = __ldg(a.val + ys + t);
+        cp_async4(s_col + t, a.col + ys + t);
+        cp_async4(s_val + t, a.val + ys + t);
     }
+    cp_async_wait_all();
     __syncwarp();
 
     // a3: the Alg. 2 walk; NR lane groups each gather one non-zero per instruction

@@ -486,6 +486,45 @@ def test_write_stats_match_alg2_counters():
             assert M.write_stats(A, sch) == (na, nr)
 
 
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+@pytest.mark.parametrize("K", [4, 16, 64, 130, 256])
+def test_kernel_write_counts_match_alg2(fixup, K):
+    """NEXT-1, Fig. 5: the counters INSIDE the segment kernel (what it wrote)
+    equal the oracle's serial Alg. 2 counters O6: issued + elided partial-row updates =
+    #atomic, complete-row stores = #regular; C is bit-exact with integer inputs."""
+    rs = np.random.RandomState(80 + K)
+    for trial in range(10):
+        g = rand_graph(rs, int(rs.randint(1, 500)), 60, 11, seed=trial)
+        A = dev(g)
+        B = G.dense_int(60, K, seed=trial)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for cost in (1, 5, 23, 200):
+            sch = M.Schedule.build(A, K, items_per_part=cost, min_parts=1)
+            C, (issued, elided, regular) = M.write_counts(A, tB(B), sch, fixup=fixup)
+            torch.cuda.synchronize()
+            _, na, nr = O.alg2_emulate(g.row_ptr, g.col_idx, g.val, B[:, :1],
+                                       sch.coord_x.cpu().numpy(), sch.coord_y.cpu().numpy())
+            assert (issued + elided, regular) == (na, nr), (trial, cost)
+            assert M.write_stats(A, sch) == (na, nr)
+            assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (trial, cost)
+
+
+def test_kernel_write_counts_full_size_reddit():
+    """The statistic at full size on the bench's workload (Reddit K=64, default plan):
+    kernel counters == O6 == mps_write_stats."""
+    g = G.workload("reddit")
+    A = dev(g)
+    sch = M.Schedule.build(A, 64)
+    B = torch.zeros((g.n, 64), device="cuda")
+    _, (issued, elided, regular) = M.write_counts(A, B, sch)
+    _, na, nr = O.alg2_emulate(g.row_ptr, g.col_idx, g.val, np.zeros((g.n, 1), np.float32),
+                               sch.coord_x.cpu().numpy(), sch.coord_y.cpu().numpy())
+    assert (issued + elided, regular) == (na, nr)
+    cx, cy = sch.coord_x.cpu().numpy(), sch.coord_y.cpu().numpy()
+    cut = np.unique(cx[(cx < g.m) & (cy > g.row_ptr[np.minimum(cx, g.m)])])
+    assert regular == g.m - len(cut)         # every row not cut is stored exactly once
+
+
 def test_validate_csr():
     g = G.workload("cora")
     assert M.validate_csr(dev(g)) == -1

@@ -21,6 +21,7 @@ from paper_conf_ispass_shangndk23_b200.api import _p, _stream
 
 KS = tuple(int(x) for x in os.environ.get("SENS_KS", "2 4 8 16 32 64 128 256").split())
 DT = 1 if os.environ.get("SENS_DTYPE", "f32") == "bf16" else 0   # B dtype code
+KS_STATS = int(os.environ.get("SENS_STATS_K", "16"))   # K of the Fig. 5 statistic + parity
 COSTS = tuple(int(x) for x in os.environ.get("SENS_COSTS", "0 64 128 256 512 1024 2048 4096").split())
 
 
@@ -76,11 +77,17 @@ def main():
                 ms = replay_ms(run)
                 row = {"graph": nm, "type": ty, "n": g.m, "nnz": g.nnz, "K": K, "cost": cost,
                        "P": P, "L": Lp, "ms": ms, "gflops": 2.0 * g.nnz * K / ms / 1e6}
-                if K == 16 and cost == 0:
+                if K == KS_STATS and cost == 0:
                     cnt = torch.empty(2, dtype=torch.int64, device="cuda")
                     L.mps_write_stats(ctypes.byref(a), _p(cx), _p(cy), P, _p(cnt), s)
                     c = cnt.cpu().tolist()
                     row["writes_atomic"], row["writes_regular"] = int(c[0]), int(c[1])
+                    # the same statistic counted inside the segment kernel (what it wrote)
+                    sch = M.Schedule(P, Lp, cx, cy)
+                    _, (iss, eli, reg) = M.write_counts(A, B, sch)
+                    row["kernel_writes"] = {"atomic_issued": iss, "atomic_elided_empty": eli,
+                                            "regular": reg}
+                    row["kernel_counts_match"] = (iss + eli, reg) == (int(c[0]), int(c[1]))
                     run()
                     torch.cuda.synchronize()
                     ref, bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B.float().cpu().numpy())
