@@ -68,6 +68,9 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP
 #define MPS_STATIC_ULCAP 4
 #endif
+#ifndef MPS_DYN_ULCAP
+#define MPS_DYN_ULCAP 0     // experiment: cap the dynamic instantiation's gathers per lane
+#endif
 #ifndef MPS_STATIC_ULCAP_MINNR
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
@@ -105,8 +108,10 @@ segment_kernel(const SegArgsT<IT> a) {
     constexpr int UL0 = (sizeof(TB) == 2 && UL00 / MPS_UL_DIV >= 2) ? UL00 / MPS_UL_DIV
                                                                     : UL00 * (DEEP ? 2 : 1);
     constexpr int UL1 = (UL0 * NR > MPS_UMAX) ? (MPS_UMAX / NR > 0 ? MPS_UMAX / NR : 1) : UL0;
-    constexpr int UL = (!DYN && NR >= MPS_STATIC_ULCAP_MINNR && UL1 > MPS_STATIC_ULCAP)
-                           ? MPS_STATIC_ULCAP : UL1;
+    constexpr int UL2 = (!DYN && NR >= MPS_STATIC_ULCAP_MINNR && UL1 > MPS_STATIC_ULCAP)
+                            ? MPS_STATIC_ULCAP : UL1;
+    constexpr int UL = (DYN && MPS_DYN_ULCAP > 0 && NR >= 2 && UL2 > MPS_DYN_ULCAP)
+                           ? MPS_DYN_ULCAP : UL2;
     constexpr int U = UL * NR;                           // non-zeros per batch
     static_assert(kCH % U == 0, "chunk must hold whole batches");
 
