@@ -57,6 +57,7 @@ def _L():
         lib.oracle_alg2_emulate.argtypes = [_i64, _p, _p, _p, _p, _i64, _i32, _p, _p, _i64,
                                             _p, _i64, _p, _p]
         lib.oracle_shard.argtypes = [_p, _i64, _i64, _i32, _p, _p, _p]
+        lib.oracle_xw_f64.argtypes = [_i64, _i64, _i32, _p, _i64, _p, _i64, _i32, _p, _i64]
         lib.oracle_shard_local.argtypes = [_i64, _p, _p, _p, _p, _i64, _i32, _i64, _i64, _i64,
                                            _i64, _p, _i64, _p]
         _lib = lib
@@ -204,6 +205,22 @@ def shard_local(row_ptr, col_idx, val, B, X, Y, g):
                             int(X[g]), int(Y[g]), int(X[g + 1]), int(Y[g + 1]),
                             _ptr(C) if C.size else None, K, _ptr(tail) if K else None)
     return C, tail
+
+
+def xw_f64(X, W, relu=False):
+    """O9 (sec. II: H' = sigma(A X W)): the combination X*W of a GCN layer, and
+    the ReLU when ``relu``, in fp64.  X: n x F, W: F x N (W itself, not its transpose),
+    any float dtype convertible to float32 exactly (bf16 values are)."""
+    X = np.ascontiguousarray(X, dtype=np.float32)
+    W = np.ascontiguousarray(W, dtype=np.float32)
+    n, F = X.shape
+    F2, N = W.shape
+    assert F == F2
+    out = np.zeros((n, N), np.float64)
+    rc = _L().oracle_xw_f64(n, F, N, _ptr(X), F, _ptr(W), N, 1 if relu else 0,
+                            _ptr(out), N)
+    assert rc == 0
+    return out
 
 
 def check(C, C_ref, bound, rel=1e-5, abs_tol=1e-7):

@@ -24,6 +24,7 @@
  *   O5 oracle_merge_walk     explicit merge of row ends and nnz      (Fig. 3 text)
  *   O6 oracle_alg2_emulate   serial Alg. 2 with write counters       (Alg. 2)
  *   O7 oracle_shard          merge-path shard bounds + tail rows     (north star stage 4)
+ *   O9 oracle_xw_f64         the combination X*W (+ ReLU) of a GCN layer (NEXT-3)
  *
  * Parity pins for every function live in tests/test_oracle_pins.py (see DESIGN.md
  * "Oracle pins").  No function here is "parity unpinned".
@@ -341,6 +342,35 @@ int oracle_shard_local(int64_t m, const int32_t *RP, const int32_t *CP, const fl
     if (Xg1 < m && Yg1 > RP[Xg1]) {
         int64_t j0 = RP[Xg1] > Yg ? RP[Xg1] : Yg;
         row_partial_sum(CP, AV, XW, ldb, K, j0, Yg1, tail);
+    }
+    return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* O9: the GCN layer's combination and activation around the aggregation,     */
+/* P:37-39 (sec. II): H' = sigma(A * (X * W)) with sigma = ReLU.  This is the */
+/* X * W (combination) half and the activation, in fp64:                      */
+/*     out[i, j] = sum_{f < F} X[i, f] * W[f, j]      (relu: max(out, 0))     */
+/* X: n x F row-major (ldx), W: F x N row-major (ldw) -- W itself, not its    */
+/* transpose -- out: n x N (ldo).  Inputs are fp32 (bf16 values are exact in  */
+/* fp32); products are exact in fp64.  OpenMP over output rows only.         */
+/* ------------------------------------------------------------------------- */
+int oracle_xw_f64(int64_t n, int64_t F, int32_t N, const float *X, int64_t ldx,
+                  const float *W, int64_t ldw, int32_t relu, double *out, int64_t ldo)
+{
+    if (n < 0 || F < 0 || N < 0) return 1;
+    int64_t i;
+#pragma omp parallel for schedule(static)
+    for (i = 0; i < n; ++i) {
+        double *o = out + i * ldo;
+        for (int32_t j = 0; j < N; ++j) o[j] = 0.0;
+        for (int64_t f = 0; f < F; ++f) {
+            const double x = (double)X[i * ldx + f];
+            const float *w = W + f * ldw;
+            for (int32_t j = 0; j < N; ++j) o[j] += x * (double)w[j];
+        }
+        if (relu)
+            for (int32_t j = 0; j < N; ++j) o[j] = o[j] > 0.0 ? o[j] : 0.0;
     }
     return 0;
 }

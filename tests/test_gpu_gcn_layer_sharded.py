@@ -31,7 +31,7 @@ def test_sharded_gcn_layer_loopback(world, N, tile):
     gen = torch.Generator().manual_seed(N)
     X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
     W = torch.randint(-1, 2, (F, N), generator=gen).to(torch.bfloat16)
-    Bref = (X.double() @ W.double()).numpy()                  # |.| <= 72: exact in bf16
+    Bref = O.xw_f64(X.float().numpy(), W.float().numpy())     # |.| <= 72: exact in bf16
     ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bref, want_bound=False)
     Xd, Wt = X.cuda(), W.t().contiguous().cuda()
     Bs = [torch.full((n, N), float("nan"), dtype=torch.bfloat16, device="cuda")
@@ -81,7 +81,7 @@ g = G.random_csr(n, n, rl, 2)
 gen = torch.Generator().manual_seed(9)
 X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
 W = torch.randint(-1, 2, (F, N), generator=gen).to(torch.bfloat16)
-Bref = (X.double() @ W.double()).numpy()
+Bref = O.xw_f64(X.float().numpy(), W.float().numpy())
 ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bref, want_bound=False)
 layer = M.ShardedGCNLayer(g.row_ptr, g.col_idx, g.val, n, F, N, rank, world, "cuda:0",
                           tile_cols=32, items_per_part=31, min_parts=1)
@@ -149,7 +149,7 @@ torch.cuda.synchronize(); dist.barrier()
 ok = True
 x0, x1 = int(layer.sh.X[rank]), int(layer.sh.X[rank + 1])
 for k in range(5):
-    Bref = (Xs[k].double() @ W.double()).numpy()
+    Bref = O.xw_f64(Xs[k].float().numpy(), W.float().numpy())
     ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bref, want_bound=False)
     ok = ok and np.array_equal(outs[k].cpu().numpy().astype(np.float64), ref[x0:x1])
 layer.close()
@@ -198,10 +198,10 @@ def test_sharded_gcn2_loopback(world):
     X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
     W1 = torch.randint(-1, 2, (F, Hd), generator=gen).to(torch.bfloat16)
     W2 = torch.randint(-1, 2, (Hd, Cd), generator=gen).to(torch.bfloat16)
-    B1 = _bf16_rne(X.double().numpy() @ W1.double().numpy())
+    B1 = _bf16_rne(O.xw_f64(X.float().numpy(), W1.float().numpy()))
     C1 = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B1, want_bound=False)
     Hh = _bf16_rne(np.maximum(C1, 0.0))
-    B2 = _bf16_rne(Hh @ W2.double().numpy())
+    B2 = _bf16_rne(O.xw_f64(Hh.astype(np.float32), W2.float().numpy()))
     ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B2, want_bound=False)
 
     def peers(N):

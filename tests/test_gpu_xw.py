@@ -3,6 +3,8 @@ import numpy as np
 import pytest
 import torch
 
+import oracle as O
+
 pytestmark = pytest.mark.gpu
 
 if torch.cuda.is_available():
@@ -24,7 +26,7 @@ def test_xw_exact_small_integers(N, F):
     X = torch.randint(-1, 2, (n, F), generator=g).to(torch.bfloat16).cuda()
     W = torch.randint(-1, 2, (F, N), generator=g).to(torch.bfloat16).cuda()
     B = M.xw_bf16(X, W.t().contiguous())
-    ref = X.double().cpu() @ W.double().cpu()
+    ref = torch.from_numpy(O.xw_f64(X.float().cpu().numpy(), W.float().cpu().numpy()))
     assert torch.equal(B.double().cpu(), ref)
 
 
@@ -37,8 +39,8 @@ def test_xw_random_within_bf16_rounding(n, F, N):
     Wt = _pad(W.t().contiguous().cuda(), ldx)
     B = M.xw_bf16(X, Wt)
     Xd, Wd = X.double().cpu(), W.double()
-    ref = Xd @ Wd
-    bound = Xd.abs() @ Wd.abs()
+    ref = torch.from_numpy(O.xw_f64(Xd.numpy(), Wd.numpy()))
+    bound = torch.from_numpy(O.xw_f64(Xd.abs().numpy(), Wd.abs().numpy()))
     err = (B.double().cpu() - ref).abs()
     # bf16 output rounding (unit roundoff 2^-8) + fp32 accumulation of F products
     assert torch.all(err <= 2.0 ** -8 * ref.abs() + 1e-5 * bound + 1e-30)
@@ -58,6 +60,6 @@ def test_xw_unaligned_feature_width_is_padded():
     X = torch.randint(-1, 2, (500, 1433), generator=g).to(torch.bfloat16)
     W = torch.randint(-1, 2, (1433, 16), generator=g).to(torch.bfloat16)
     B = M.xw_bf16(X.cuda(), W.t().contiguous().cuda())
-    ref = X.double() @ W.double()
+    ref = torch.from_numpy(O.xw_f64(X.float().numpy(), W.float().numpy()))
     # |sum| <= 1433: bf16 rounds, compare within one bf16 ulp of the exact integer
     assert torch.all((B.double().cpu() - ref).abs() <= ref.abs() * 2.0 ** -8)

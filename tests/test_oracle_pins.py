@@ -384,3 +384,58 @@ def test_o7_owner_consumes_row_end():
             shard = int(np.searchsorted(D, step, side="left")) - 1  # D_g < step <= D_{g+1}
             owner = max(gg for gg in range(world) if X[gg] <= r)
             assert shard == owner
+
+
+def test_o4_plan_thread_floor_p139():
+    """"When the computed threads are below a threshold (e.g., 1024), the total
+    thread count is set to the threshold value" -- "the merge path cost is decreased to
+    ensure a minimum number of threads".  Checked by brute force: with the threshold in
+    force the thread count equals it and the items per thread are the SMALLEST count
+    that lets 1024 threads cover the merge path (found by search, not by formula), never
+    above the requested cost; above the threshold the cost is kept.  The partition of a
+    random CSR of that size then covers the merge path with segments of <= L items."""
+    rs = np.random.RandomState(139)
+    for M_items, cost in [(10_000, 20), (1_500, 50), (1023, 1), (13_264, 64), (100_000, 64)]:
+        m = M_items // 3
+        nnz = M_items - m
+        P, L = O.plan(m, nnz, cost, 1024)
+        threads_from_cost = -(-M_items // cost)           # merge_items / cost (P:137)
+        if threads_from_cost < 1024:
+            assert P == 1024
+            assert L == min(l for l in range(1, cost + 1) if 1024 * l >= M_items)
+            assert L <= cost                                # the cost is decreased
+        else:
+            assert P == threads_from_cost and L <= cost
+        rl = rs.multinomial(nnz, np.ones(m) / m).astype(np.int32)
+        rp = np.concatenate([[0], np.cumsum(rl)]).astype(np.int32)
+        cx, cy = O.partition(rp, P, L)
+        d = cx.astype(np.int64) + cy
+        assert d[0] == 0 and d[-1] == M_items and np.all(np.diff(d) >= 0)
+        assert np.all(np.diff(d) <= L)
+
+
+def test_o9_xw_pins():
+    """O9 (combination X*W and the ReLU of sigma(A X W), P:37-39) pinned by: identity W;
+    one-hot rows of X selecting rows of W (catches a transposed W); all-ones X giving the
+    column sums of W (np.sum); a pure-Python triple loop on a tiny case; ReLU as the
+    elementwise max with 0 of that brute force; rank-1 X = u v^T giving u (v^T W)."""
+    rs = np.random.RandomState(9)
+    X = rs.randn(7, 5).astype(np.float32)
+    assert np.array_equal(O.xw_f64(X, np.eye(5, dtype=np.float32)), X.astype(np.float64))
+    W = rs.randn(5, 3).astype(np.float32)
+    E = np.eye(5, dtype=np.float32)[[4, 0, 2]]
+    assert np.array_equal(O.xw_f64(E, W), W[[4, 0, 2]].astype(np.float64))
+    Wi = rs.randint(-5, 6, size=(9, 4)).astype(np.float32)
+    assert np.array_equal(O.xw_f64(np.ones((3, 9), np.float32), Wi),
+                          np.tile(Wi.astype(np.float64).sum(0), (3, 1)))
+    Xs = rs.randint(-3, 4, size=(4, 6)).astype(np.float32)
+    Ws = rs.randint(-3, 4, size=(6, 5)).astype(np.float32)
+    bf = np.array([[sum(float(Xs[i, f]) * float(Ws[f, j]) for f in range(6)) for j in range(5)]
+                   for i in range(4)])
+    assert np.array_equal(O.xw_f64(Xs, Ws), bf)
+    assert np.array_equal(O.xw_f64(Xs, Ws, relu=True), np.where(bf > 0, bf, 0.0))
+    u = rs.randint(-2, 3, size=8).astype(np.float32)
+    v = rs.randint(-2, 3, size=6).astype(np.float32)
+    vW = [sum(float(v[f]) * float(Ws[f, j]) for f in range(6)) for j in range(5)]
+    assert np.array_equal(O.xw_f64(np.outer(u, v).astype(np.float32), Ws),
+                          np.array([[float(ui) * x for x in vW] for ui in u]))
