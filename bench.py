@@ -732,6 +732,38 @@ def main():
             # ncu DRAM bytes of one launch (one column tile) over the live launch time
             per_launch_s = t_seg * 1e-3 / max(1, n_tiles(g.n, K, b_elt, l2))
             roof["dram_frac_of_peak_ncu_bytes"] = traffic / per_launch_s / 1e9 / hbm_peak
+    # The workload's own gather stream replayed alone (tools/gather_replay.cu): the B-row
+    # gathers of every non-zero in CSR order (row col_idx[j] of each column tile), read
+    # with nothing else in the way, L2 flushed first.  Its time is the attainable time of
+    # the kernel's dominant traffic on this box, with the L2-hit / DRAM-miss mix the real
+    # column pattern produces; roofline.peak is the algorithmic byte rate at that time.
+    row_bytes = tile_cols * b_elt
+    if world == 1 and not args.no_l2_probe and row_bytes in (64, 128, 256, 512) \
+            and online.path != L.MPS_PATH_SMALL_FUSED:
+        try:
+            import __graft_entry__
+            gr = ctypes.CDLL(__graft_entry__.build_gather_replay())
+            gms, gby = ctypes.c_float(), ctypes.c_double()
+            rc = gr.gather_replay(_p(A.col_idx), ctypes.c_int64(g.nnz), _p(Bd),
+                                  ctypes.c_int32(row_bytes), ctypes.c_int64(K * b_elt),
+                                  ctypes.c_int32(3), ctypes.byref(gms), ctypes.byref(gby))
+            torch.cuda.synchronize(dev)
+            if rc == 0 and gms.value > 0:
+                tiles = n_tiles(g.n, K, b_elt, l2)
+                t_rep = gms.value * tiles                       # every column tile
+                roof["attainable"] = {
+                    "what": "gather replay: the B-row gathers of the workload's own col_idx "
+                            "stream alone, %d x %d-B rows per non-zero, L2 flushed" % (
+                                tiles, row_bytes),
+                    "replay_ms": t_rep, "segment_ms": t_seg,
+                    "gather_gbs": gby.value * tiles / (t_rep * 1e-3) / 1e9,
+                    "frac": t_rep / t_seg}
+                roof["units_frac_against"] = {"l2_probe": (seg_gbs / l2_peak) if l2_peak else None,
+                                              "hbm_peak": seg_gbs / hbm_peak}
+                roof.update({"peak": seg_bytes / (t_rep * 1e-3) / 1e9, "frac": t_rep / t_seg,
+                             "peak_source": "gather replay of this workload (roofline.attainable)"})
+        except Exception as e:  # pragma: no cover
+            roof["attainable_error"] = str(e)[:200]
 
     # cuSPARSE on the same A, B (reference point; not the product)
     cus = None
