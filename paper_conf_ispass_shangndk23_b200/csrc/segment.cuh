@@ -610,13 +610,14 @@ static bool dynamic_claims() {
     return e ? atoi(e) != 0 : true;
 }
 
-// Occupancy of one instantiation, per device (the carveout hint is a per-device
-// function attribute).  Idempotent, so concurrent first calls from several host
-// threads only repeat the same query.
+// Occupancy of one instantiation, per device (the carveout / dynamic shared memory are
+// per-device function attributes).  `cache` is the calling instantiation's own (a
+// static of launch_seg<...>): the kernels share one function-pointer type, so a cache
+// keyed on the type alone would hand one kernel's occupancy to all.  Idempotent, so
+// concurrent first calls from several host threads only repeat the same query.
 template <typename KFn>
-static cudaError_t seg_blocks_per_sm(KFn kstatic, KFn kdyn, int *out, size_t dsm_st = 0,
-                                     size_t dsm_dy = 0) {
-    static std::atomic<int> cache[64];
+static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic, KFn kdyn,
+                                     int *out, size_t dsm_st = 0, size_t dsm_dy = 0) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -662,8 +663,9 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     // is not guaranteed: each gets its own)
     const size_t ring_st = ASYNC ? seg_ring_bytes<W, V, NR, TB, false>() : 0;
     const size_t ring_dy = ASYNC ? seg_ring_bytes<W, V, NR, TB, true>() : 0;
+    static std::atomic<int> occ_cache[64];      // per instantiation, per device
     int blocks_per_sm = 0;
-    cudaError_t e = seg_blocks_per_sm(kst, kdy, &blocks_per_sm, ring_st, ring_dy);
+    cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, &blocks_per_sm, ring_st, ring_dy);
     if (e != cudaSuccess) return e;
     const int64_t warps_per_block = kBlock / 32;
     int64_t need = (a.P + warps_per_block - 1) / warps_per_block;

@@ -224,7 +224,11 @@ constexpr int kXpMaxStages = 8;
 __global__ void __launch_bounds__(kXpThreads, 1)
 xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
                      const __grid_constant__ CUtensorMap map_w, int64_t n, int F, int N,
-                     int stages, const XwDst dst, int64_t ldb, int staged, int nsplit) {
+                     int stages, const XwDst dst, int64_t ldb, int staged, int nsplit,
+                     int wstream) {
+    // wstream = 1: W is NOT resident -- each ring stage carries the X chunk AND the
+    // matching 64-wide chunk of W (re-read from L2 for every tile), for W too large for
+    // shared memory (Reddit K=256: W = 256 x 602 bf16 = 308 KB)
     // N = the column slice this CTA computes; nsplit slices of W / B are spread over
     // consecutive CTAs (W too large for shared memory as a whole, or TMEM for 2 CTAs)
     const int slice = (int)(blockIdx.x % (unsigned)nsplit);
@@ -235,9 +239,10 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
     const int nk = (F + kXwBK - 1) / kXwBK;
     const uint32_t a_bytes = kXwBM * kXwBK * 2;            // 16 KB per X stage
     const uint32_t wchunk = (uint32_t)N * kXwBK * 2;        // one 64-wide chunk of W
+    const uint32_t stage_bytes = a_bytes + (wstream ? wchunk : 0u);
     uint8_t *sW = base;
-    uint8_t *sA = base + (size_t)nk * wchunk;
-    uint64_t *full = (uint64_t *)(sA + (size_t)stages * a_bytes);
+    uint8_t *sA = base + (wstream ? (size_t)0 : (size_t)nk * wchunk);
+    uint64_t *full = (uint64_t *)(sA + (size_t)stages * stage_bytes);
     uint64_t *empty = full + kXpMaxStages;
     uint64_t *acc_full = empty + kXpMaxStages;              // [2]
     uint64_t *acc_empty = acc_full + 2;                     // [2]
@@ -276,20 +281,27 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
 
     if (warp == 0) {
         if (lane == 0) {
-            // ---- TMA producer: W once, then the X ring across this CTA's tiles ----
-            mbar_arrive_expect_tx(w_full, (uint32_t)nk * wchunk);
-            for (int kb = 0; kb < nk; ++kb)
-                tma_load_2d(smem_u32(sW + (size_t)kb * wchunk), &map_w, kb * kXwBK, col_off,
-                            smem_u32(w_full));
+            // ---- TMA producer: W once (resident), then the X ring across this CTA's
+            //      tiles; streamed W: every stage also carries its W chunk ----
+            if (!wstream) {
+                mbar_arrive_expect_tx(w_full, (uint32_t)nk * wchunk);
+                for (int kb = 0; kb < nk; ++kb)
+                    tma_load_2d(smem_u32(sW + (size_t)kb * wchunk), &map_w, kb * kXwBK, col_off,
+                                smem_u32(w_full));
+            }
             uint32_t it = 0;
             for (int64_t t = t0; t < ntiles; t += tstride) {
                 for (int kb = 0; kb < nk; ++kb, ++it) {
                     const uint32_t s = it % (uint32_t)stages;
                     if (it >= (uint32_t)stages)
                         mbar_wait_u32(smem_u32(&empty[s]), ((it / stages) - 1) & 1);
-                    mbar_arrive_expect_tx(&full[s], a_bytes);
-                    tma_load_2d(smem_u32(sA + (size_t)s * a_bytes), &map_x, kb * kXwBK,
-                                (int)(t * kXwBM), smem_u32(&full[s]));
+                    uint8_t *st = sA + (size_t)s * stage_bytes;
+                    mbar_arrive_expect_tx(&full[s], stage_bytes);
+                    tma_load_2d(smem_u32(st), &map_x, kb * kXwBK, (int)(t * kXwBM),
+                                smem_u32(&full[s]));
+                    if (wstream)
+                        tma_load_2d(smem_u32(st + a_bytes), &map_w, kb * kXwBK, col_off,
+                                    smem_u32(&full[s]));
                 }
             }
         }
@@ -297,7 +309,7 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
         if (lane == 0) {
             // ---- MMA issuer ----
             const uint32_t idesc = instr_desc_bf16(N);
-            mbar_wait_u32(smem_u32(w_full), 0);
+            if (!wstream) mbar_wait_u32(smem_u32(w_full), 0);
             uint32_t it = 0, i = 0;
             for (int64_t t = t0; t < ntiles; t += tstride, ++i) {
                 const uint32_t acc = i & 1u, use = i >> 1;
@@ -308,8 +320,10 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
                     const uint32_t s = it % (uint32_t)stages;
                     mbar_wait_u32(smem_u32(&full[s]), (it / stages) & 1);
                     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-                    const uint64_t da = smem_desc_sw128(smem_u32(sA + (size_t)s * a_bytes));
-                    const uint64_t db = smem_desc_sw128(smem_u32(sW + (size_t)kb * wchunk));
+                    uint8_t *st = sA + (size_t)s * stage_bytes;
+                    const uint64_t da = smem_desc_sw128(smem_u32(st));
+                    const uint64_t db = smem_desc_sw128(
+                        smem_u32(wstream ? st + a_bytes : sW + (size_t)kb * wchunk));
 #pragma unroll
                     for (int k = 0; k < kXwBK / 16; ++k) {
                         const uint32_t accum = (kb > 0 || k > 0) ? 1u : 0u;
@@ -504,6 +518,50 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
         const char *e = getenv("MPS_XW_SPLIT");
         return e ? atoi(e) : 0;
     }();
+    // MPS_XW_WSTREAM: 1 = stream W through the ring even when it fits (A/B), 0 = never
+    static const int wstream_env = [] {
+        const char *e = getenv("MPS_XW_WSTREAM");
+        return e ? atoi(e) : -1;
+    }();
+    static const int staged = [] {
+        const char *e = getenv("MPS_XW_STAGED");
+        return e ? atoi(e) : 1;
+    }();
+    const size_t xw_budget = 227u << 10, xw_fixed = 1024 + 512 + 8 * 32 * 64;
+    auto set_persist_attr = [&]() -> cudaError_t {
+        // function attributes are per device: set once for each
+        static bool pattr[64] = {false};
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) dev = 0;
+        if (!pattr[dev]) {
+            cudaError_t e = cudaFuncSetAttribute(xw_persistent_kernel,
+                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                 (int)xw_budget);
+            if (e != cudaSuccess) return e;
+            pattr[dev] = true;
+        }
+        return cudaSuccess;
+    };
+    // streamed-W persistent kernel: the whole N per CTA (TMEM 2 x N <= 512 columns), stages
+    // of X chunk + W chunk; two CTAs per SM when three stages fit in half the budget
+    auto launch_wstream = [&]() -> cudaError_t {
+        const size_t stage_bytes = (size_t)kXwBM * kXwBK * 2 + (size_t)N * kXwBK * 2;
+        int per_sm = ((113u << 10) - xw_fixed) / stage_bytes >= 3 ? 2 : 1;
+        if (2 * 2 * N > 512) per_sm = 1;
+        int stages = (int)(((per_sm == 2 ? (113u << 10) : xw_budget) - xw_fixed) / stage_bytes);
+        stages = stages > max_stages ? max_stages : stages;
+        if (stages < 2) return cudaErrorNotSupported;
+        cudaError_t e = set_persist_attr();
+        if (e != cudaSuccess) return e;
+        const size_t smem = xw_fixed + (size_t)stages * stage_bytes;
+        const int64_t ntiles = (n + kXwBM - 1) / kXwBM;
+        int64_t grid = (int64_t)num_sms() * per_sm;
+        if (grid > ntiles) grid = ntiles;
+        xw_persistent_kernel<<<(unsigned)grid, kXpThreads, smem, s>>>(
+            mx, mw, n, (int)F, N, stages, dst, ldb, staged, 1, 1);
+        return cudaGetLastError();
+    };
+    if (persist && wstream_env == 1) return launch_wstream();
     if (persist) {
         // Choose the column slice width Nh of W / B one CTA owns (nsplit = N / Nh slices
         // on consecutive CTAs; X tiles are then read once per slice, the repeats from L2).
@@ -535,30 +593,23 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
             stages = stages > max_stages ? max_stages : stages;
             stages = stages < 2 ? 2 : stages;
             const size_t smem = fixed + wb(nh) + (size_t)stages * a_bytes;
-            // function attributes are per device: set once for each
-            static bool pattr[64] = {false};
-            int dev = 0;
-            if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) dev = 0;
-            if (!pattr[dev]) {
-                cudaError_t e = cudaFuncSetAttribute(xw_persistent_kernel,
-                                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                     (int)budget);
-                if (e != cudaSuccess) return e;
-                pattr[dev] = true;
-            }
+            cudaError_t ea = set_persist_attr();
+            if (ea != cudaSuccess) return ea;
             CUtensorMap mws;
             if (nh != N && !make_map(&mws, Wt, N, F, ldw, nh)) return cudaErrorNotSupported;
             const int64_t ntiles = (n + kXwBM - 1) / kXwBM;
             int64_t grid = (int64_t)num_sms() * per_sm / nsplit * nsplit;
             if (grid > ntiles * nsplit) grid = ntiles * nsplit;
             if (grid < nsplit) grid = nsplit;
-            static const int staged = [] {
-                const char *e = getenv("MPS_XW_STAGED");
-                return e ? atoi(e) : 1;
-            }();
             xw_persistent_kernel<<<(unsigned)grid, kXpThreads, smem, s>>>(
-                mx, nh == N ? mw : mws, n, (int)F, nh, stages, dst, ldb, staged, nsplit);
+                mx, nh == N ? mw : mws, n, (int)F, nh, stages, dst, ldb, staged, nsplit, 0);
             return cudaGetLastError();
+        }
+        // W does not fit in shared memory: stream it through the ring with X (the
+        // one-tile-per-CTA kernel below reached 46% of HBM on Reddit K=256)
+        if (wstream_env != 0) {
+            const cudaError_t e = launch_wstream();
+            if (e != cudaErrorNotSupported) return e;
         }
     }
     // stages: enough to cover the reduction, but small enough that >= 2 CTAs share an SM

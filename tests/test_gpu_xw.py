@@ -63,3 +63,34 @@ def test_xw_unaligned_feature_width_is_padded():
     ref = torch.from_numpy(O.xw_f64(X.float().numpy(), W.float().numpy()))
     # |sum| <= 1433: bf16 rounds, compare within one bf16 ulp of the exact integer
     assert torch.all((B.double().cpu() - ref).abs() <= ref.abs() * 2.0 ** -8)
+
+
+def test_xw_streamed_w_when_w_does_not_fit():
+    """Reddit K=256's combination (F = 602, N = 256: W = 308 KB > shared memory): the
+    persistent kernel streams W chunks through the ring with X.  Within bf16 rounding of
+    the fp64 oracle O9."""
+    g = torch.Generator(device="cpu").manual_seed(602)
+    n, F, N = 4097, 602, 256
+    ldx = (F + 7) // 8 * 8
+    X = _pad(torch.randn(n, F, generator=g).to(torch.bfloat16).cuda(), ldx)
+    W = (torch.randn(F, N, generator=g) / F ** 0.5).to(torch.bfloat16)
+    Wt = _pad(W.t().contiguous().cuda(), ldx)
+    B = M.xw_bf16(X, Wt)
+    Xd, Wd = X.double().cpu(), W.double()
+    ref = torch.from_numpy(O.xw_f64(Xd.numpy(), Wd.numpy()))
+    bound = torch.from_numpy(O.xw_f64(Xd.abs().numpy(), Wd.abs().numpy()))
+    err = (B.double().cpu() - ref).abs()
+    assert torch.all(err <= 2.0 ** -8 * ref.abs() + 1e-5 * bound + 1e-30)
+
+
+def test_xw_streamed_w_forced_exact():
+    """MPS_XW_WSTREAM=1 (W streamed even where it fits): the small-integer shapes stay
+    bit-exact (the knob is read once per process: run in a subprocess)."""
+    import os, subprocess, sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, MPS_XW_WSTREAM="1")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-p", "no:cacheprovider",
+                        os.path.join(root, "tests", "test_gpu_xw.py"), "-k",
+                        "exact_small_integers"], env=env, capture_output=True, text=True,
+                       timeout=600, cwd=root)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]

@@ -101,6 +101,47 @@ __global__ void __launch_bounds__(256) l2_stream_lean(const uint4 *__restrict__ 
     if (acc == 0x9e3779b9u) sink[0] = acc;
 }
 
+// mode 4: lean random gathers through asynchronous copies (cp.async 16 B, LDGSTS) into
+// a per-warp shared-memory ring of 2 batches: each lane issues 16 copies for batch b+1,
+// then waits for batch b (cp.async.wait_group 1) and reads its own 16 B back (LDS) --
+// the landing path a register-free pipelined gather would use.
+template <int U>
+__global__ void __launch_bounds__(256) l2_gather_async(const uint4 *__restrict__ tab,
+                                                       uint32_t shift, uint32_t row16,
+                                                       int iters, uint32_t *sink) {
+    __shared__ uint4 ring[8][2][U][32];
+    const uint32_t warp_in = threadIdx.x >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t grp = lane / row16, lr = lane % row16;
+    const uint32_t warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    uint32_t x = mix32(warp * 0x9E3779B9u + grp * 0x85ebca6bu + 7u);
+    uint32_t acc = 0;
+    auto issue = [&](int slot) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            x = x * 1664525u + 1013904223u;
+            const uint4 *src = tab + (uint64_t)(x >> shift) * row16 + lr;
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
+                         :: "r"((uint32_t)__cvta_generic_to_shared(&ring[warp_in][slot][u][lane])),
+                            "l"(src) : "memory");
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    issue(0);
+    for (int it = 0; it < iters; ++it) {
+        const int cur = it & 1;
+        issue(cur ^ 1);
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const uint4 v = ring[warp_in][cur][u][lane];
+            acc ^= v.x ^ v.y ^ v.z ^ v.w;
+        }
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    if (acc == 0x9e3779b9u) sink[0] = acc;
+}
+
 // mode 0: random row gathers (row_bytes in {16..512}); mode 1: streaming read;
 // mode 2: lean random gathers (power-of-two rows); mode 3: lean streaming read.
 // Returns 0 on success; *gbs = best bytes read / time over the tried grid shapes.
@@ -135,6 +176,7 @@ extern "C" int l2_probe_read_gbs2(int64_t bytes, int32_t row_bytes, int32_t mode
         const int passes = 20;
         if (mode == 0) l2_gather<8><<<grid, 256>>>(buf, nrows, row16, 20, sink);
         else if (mode == 2) l2_gather_lean<16><<<grid, 256>>>(buf, shift, row16, 10, sink);
+        else if (mode == 4) l2_gather_async<6><<<grid, 256>>>(buf, shift, row16, 10, sink);
         else l2_stream<<<grid, 256>>>(buf, n16, 1, sink);       // make it resident
         for (int rep = 0; rep < 3; ++rep) {
             cudaEventRecord(e0);
@@ -145,6 +187,9 @@ extern "C" int l2_probe_read_gbs2(int64_t bytes, int32_t row_bytes, int32_t mode
             } else if (mode == 2) {
                 l2_gather_lean<16><<<grid, 256>>>(buf, shift, row16, iters / 2, sink);
                 moved = (double)grid * 256 * 16 * 16 * (iters / 2);
+            } else if (mode == 4) {
+                l2_gather_async<6><<<grid, 256>>>(buf, shift, row16, iters, sink);
+                moved = (double)grid * 256 * 16 * 6 * (iters + 1);
             } else if (mode == 3) {
                 if (steps == 0) break;
                 l2_stream_lean<8><<<grid, 256>>>(buf, (uint32_t)(steps * 8ull * st), passes, sink);
