@@ -173,6 +173,10 @@ inline int64_t seg_dynamic_min_parts() { return (int64_t)4 * 2 * (kBlock / 32) *
 __device__ __forceinline__ void count_write(unsigned long long *wstat, int lane, int k) {
     if (wstat != nullptr && lane == 0) atomicAdd(wstat + k, 1ull);
 }
+template <bool ON>
+__device__ __forceinline__ void count_write_if(unsigned long long *wstat, int lane, int k) {
+    if constexpr (ON) count_write(wstat, lane, k);
+}
 __device__ __forceinline__ int ld_stream_i32(const int32_t *p) {
     int v;
     asm volatile("ld.global.cs.s32 %0, [%1];" : "=r"(v) : "l"(p));

@@ -374,18 +374,18 @@ segment_kernel(const SegArgsT<IT> a) {
                         write_row((r == a.tail_row) ? a.tail
                                                     : a.C + ((int64_t)r - a.row_base) * a.ldc,
                                   true);
-                        count_write(a.wstat, lane, 0);
+                        count_write_if<!DYN>(a.wstat, lane, 0);
                     } else {
-                        count_write(a.wstat, lane, 1);   // empty piece: the add is elided
+                        count_write_if<!DYN>(a.wstat, lane, 1);   // empty piece: the add is elided
                     }
                 } else {
                     write_row(a.rec + ((int64_t)seg * 2) * a.kpad, false);
-                    count_write(a.wstat, lane, 0);
+                    count_write_if<!DYN>(a.wstat, lane, 0);
                 }
             } else {
                 // complete row (line 15): plain store, no initialisation of C needed
                 write_row(a.C + ((int64_t)r - a.row_base) * a.ldc, false, a.relu != 0);
-                count_write(a.wstat, lane, 2);
+                count_write_if<!DYN>(a.wstat, lane, 2);
             }
 #pragma unroll
             for (int s = 0; s < V; ++s)
@@ -488,7 +488,9 @@ segment_kernel(const SegArgsT<IT> a) {
                         cid[i] = (j >= ys && j < ye) ? cid[i] : 0u;
                     }
                 }
-                if (hot == nullptr) {
+                // (the hot-row bitmap exists in the static instantiation only: the launcher
+                // runs that one when a bitmap is passed)
+                if (DYN || hot == nullptr) {
 #pragma unroll
                     for (int i = 0; i < UL; ++i)
 #pragma unroll
@@ -598,7 +600,7 @@ segment_kernel(const SegArgsT<IT> a) {
                           true);
             else
                 write_row(a.rec + ((int64_t)seg * 2 + (single ? 0 : 1)) * a.kpad, false);
-            count_write(a.wstat, lane, 0);
+            count_write_if<!DYN>(a.wstat, lane, 0);
         }
     }
     if (a.mail.on) tail_mail_epilogue(a.mail);   // a6 tail exchange (last CTA, last tile)
@@ -638,10 +640,16 @@ static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic,
         if (e != cudaSuccess) return e;
     }
     if (dsm_st > 0 || dsm_dy > 0) {
+        // the ASYNC ring: two CTAs of ~97 KB need the maximum shared-memory carveout
         e = cudaFuncSetAttribute(kstatic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm_st);
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(kdyn, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)dsm_dy);
+        if (e == cudaSuccess && carve < 0)
+            e = cudaFuncSetAttribute(kstatic, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                     100);
+        if (e == cudaSuccess && carve < 0)
+            e = cudaFuncSetAttribute(kdyn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
         if (e != cudaSuccess) return e;
     }
     int bps = 0;
@@ -677,7 +685,10 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     // 1-6% faster); at 1-3 per warp the opening burst of claims on one counter costs more
     // than the balance gains (Table-II graphs, profiles/r01/dynamic_claims/).  The counter
     // (a.claim) lives in the caller's workspace and is zero when the kernel starts.
-    const bool dyn = a.claim != nullptr && a.P >= 4 * grid * warps_per_block && dynamic_claims();
+    // (the Fig. 5 write counters exist in the static instantiation only: a counting
+    // launch runs it, and the dynamic kernel of the large graphs carries no counting code)
+    const bool dyn = a.claim != nullptr && a.wstat == nullptr && a.hot == nullptr &&
+                     a.P >= 4 * grid * warps_per_block && dynamic_claims();
     // launched with programmatic stream serialization (PDL): the CTAs may be scheduled
     // as the previous kernel's CTAs retire, hiding the launch gap (tens of percent of a
     // small graph's step); griddepcontrol.wait in the kernel keeps the data dependency.

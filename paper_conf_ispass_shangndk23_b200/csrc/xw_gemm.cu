@@ -574,7 +574,10 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
         const size_t budget = 227u << 10, half_budget = 113u << 10;
         auto wb = [&](int nh) { return (size_t)nkp * nh * kXwBK * 2; };
         int nh = 0, per_sm = 0;
-        for (int d = 1; d <= 4 && nh == 0; d *= 2)
+        // slices (d > 1) only when streaming W is switched off (MPS_XW_WSTREAM=0): the
+        // streamed-W kernel beat them on Reddit K=256 (0.098 vs 0.139 ms, r02k)
+        const int dmax = (wstream_env == 0 || force_split > 1) ? 4 : 1;
+        for (int d = 1; d <= dmax && nh == 0; d *= 2)
             for (int pass = 0; pass < 2 && nh == 0; ++pass) {
                 const int c = N / d;
                 if (N % d || c % 16) continue;

@@ -376,8 +376,9 @@ def test_gcn2_tcgen05_combination():
     # layer 1: B1 = bf16(X) * bf16(W1) in fp32, rounded to bf16, checked vs fp64
     Xb, W1b = X.to(torch.bfloat16).double().cpu(), W1.to(torch.bfloat16).double().cpu()
     B1 = M.xw_bf16(X.to(torch.bfloat16), net.W1t)
-    ref = Xb @ W1b
-    assert torch.all((B1.double().cpu() - ref).abs() <= 2 ** -8 * ref.abs() + 1e-5 * (Xb.abs() @ W1b.abs()))
+    ref = torch.from_numpy(O.xw_f64(Xb.numpy(), W1b.numpy()))            # O9
+    bnd = torch.from_numpy(O.xw_f64(Xb.abs().numpy(), W1b.abs().numpy()))
+    assert torch.all((B1.double().cpu() - ref).abs() <= 2 ** -8 * ref.abs() + 1e-5 * bnd)
     # aggregation on exactly that bf16 B1, with the fused ReLU
     ref1, bnd1 = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B1.float().cpu().numpy())
     r = O.check(net.H.cpu().numpy(), np.maximum(ref1, 0), bnd1)
