@@ -667,17 +667,21 @@ def main():
         y0, y1 = int(sh.Y[rank]), int(sh.Y[rank + 1])
         seg_bytes = alg_bytes(sh.rows, y1 - y0, K, b_elt)
     seg_gbs = seg_bytes / (t_seg * 1e-3) / 1e9
-    traffic = None
+    traffic = None          # ncu DRAM bytes per launch of the segment kernel
     units = None
     prof = os.path.join(ROOT, "profiles", "traffic.json")
     key = "%s-k%d-%s-%s" % (name, K, args.dtype, "atomic" if args.fixup == "auto" else args.fixup)
     if os.path.exists(prof) and world == 1:
         with open(prof) as f:
             tj = json.load(f)
-            traffic = tj.get(key)
+            traffic_step = tj.get(key)          # DRAM bytes of all column tiles of a step
+            if isinstance(traffic_step, (int, float)):
+                # per launch, like `achieved` (one launch = one column tile)
+                traffic = int(traffic_step / max(1, n_tiles(g.n, K, b_elt, l2)))
             u = tj.get("_units", {}).get(key)
             if u:   # ncu of the same kernel: which unit binds (B in L2 -> L2, else DRAM)
-                units = dict(u, source="ncu --set full, profiles/r01 (traffic.json)",
+                units = dict(u, source="ncu --set full (profiles/traffic.json: %s)"
+                             % tj.get("_note", "")[:60],
                              note=("B fits in L2: the algorithmic-byte fraction exceeds 1; "
                                    "the binding unit is L2 (lts_throughput_pct)")
                              if b_elt * g.n * K <= 0.5 * l2 else

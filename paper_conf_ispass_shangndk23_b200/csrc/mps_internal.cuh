@@ -371,7 +371,9 @@ __device__ __forceinline__ void cp_async_wait_all() {
 }
 // 16-B asynchronous copy with an L2 cache policy (the B-row gathers: evict_last)
 __device__ __forceinline__ void cp_async16_l2(void *dst_smem, const void *src, uint64_t pol) {
-    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;"
+    // explicit src-size (16): with only the policy after cp-size, the fourth operand is
+    // taken as src-size (illegal instruction / partial copies)
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, 16, %2;"
                  :: "r"(smem_u32(dst_smem)), "l"(src), "l"(pol) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() {

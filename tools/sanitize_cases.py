@@ -24,7 +24,8 @@ def run():
             B = G.dense_int(300, K, seed=K)
             ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
             Bt = torch.from_numpy(B).cuda().to(dt)
-            for fixup in ("atomic", "carry"):
+            # "auto": the one-launch small-graph path (small.cu) + carry reduction
+            for fixup in ("atomic", "carry", "auto"):
                 for cost in (7, 64, 2048):
                     C = M.spmm(A, Bt, fixup=fixup, items_per_part=cost, min_parts=1)
                     torch.cuda.synchronize()
