@@ -236,14 +236,6 @@ int64_t host_diag_x(const IT *rp, int64_t m, int64_t nnz, int64_t d) {
     return lo - 1;
 }
 
-// When the cp.async-pipelined gathers run (default, no MPS_ASYNC): decided from
-// measurements (profiles/r02/async_gathers.md).
-template <typename IT>
-bool async_rule(const mps::SegArgsT<IT> &a, int32_t dt, int32_t kt) {
-    (void)a; (void)dt; (void)kt;
-    return false;
-}
-
 // Run a3 (+ a4 carry reduction) over all column tiles for a ready schedule.
 // claims: the per-tile claim counters (workspace; NULL: static segment assignment);
 // claims_zeroed: a kernel earlier on the stream already zeroed them, else they are
@@ -280,16 +272,6 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
         int V, NR;
         tile_geometry(kt, v.W, &V, &NR);
         a.deep = v.deep && kt == 64 ? 1 : 0;
-        // cp.async-pipelined gathers (segment.cuh ASYNC): MPS_ASYNC=1 forces them where
-        // the instantiation exists (16-B lanes, int32 indices, no hot-row bitmap, not
-        // the deep-gather kernel); default: the measured rule (async_rule)
-        static const int async_env = [] {
-            const char *e = getenv("MPS_ASYNC");
-            return e ? atoi(e) : -1;
-        }();
-        a.async_gather = (a.hot == nullptr && !a.deep &&
-                          (async_env == 1 || (async_env < 0 && async_rule(base, dt, kt))))
-                             ? 1 : 0;
         mps::SegArgsT<IT> seg_only = a;
         seg_only.mail.on = 0;
         MPS_CUDA(mps::launch_segments(fix == mps::FIX_CARRY ? seg_only : a, dt, v.W, V, NR, fix,

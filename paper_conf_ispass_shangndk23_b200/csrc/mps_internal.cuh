@@ -78,7 +78,6 @@ struct SegArgsT {
     unsigned *claim;     // dynamic segment claims: this column tile's counter in the caller's
                          // workspace, zero when the kernel starts (NULL: static assignment)
     int32_t deep;        // 1: deep-gather instantiation (fp32, 64-column tile, DRAM-bound B)
-    int32_t async_gather;       // 1: cp.async-pipelined B gathers (16-B lanes, int32 indices)
     unsigned long long *wstat;  // Fig. 5 counters of what the kernel wrote (NULL: off):
                                 // [0] partial-row updates (atomic / carry record),
                                 // [1] empty partial start pieces whose add was elided,
@@ -369,21 +368,6 @@ __device__ __forceinline__ void cp_async8(void *dst_smem, const void *src) {
 __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.wait_all;" ::: "memory");
 }
-// 16-B asynchronous copy with an L2 cache policy (the B-row gathers: evict_last)
-__device__ __forceinline__ void cp_async16_l2(void *dst_smem, const void *src, uint64_t pol) {
-    // explicit src-size (16): with only the policy after cp-size, the fourth operand is
-    // taken as src-size (illegal instruction / partial copies)
-    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, 16, %2;"
-                 :: "r"(smem_u32(dst_smem)), "l"(src), "l"(pol) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() {
-    asm volatile("cp.async.commit_group;" ::: "memory");
-}
-// all but the most recent commit group of this thread have landed
-__device__ __forceinline__ void cp_async_wait_group1() {
-    asm volatile("cp.async.wait_group 1;" ::: "memory");
-}
-
 // global -> shared bulk copy of `bytes` (multiple of 16, both addresses 16-B aligned),
 // completion counted on `bar`; L2 evict_first (streamed once).
 __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t bytes,

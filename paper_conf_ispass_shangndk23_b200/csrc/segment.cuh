@@ -106,21 +106,9 @@ __host__ __device__ constexpr int seg_ul() {
                             ? MPS_STATIC_ULCAP : UL1;
     return (DYN && MPS_DYN_ULCAP > 0 && NR >= 2 && UL2 > MPS_DYN_ULCAP) ? MPS_DYN_ULCAP : UL2;
 }
-// dynamic shared memory of the ASYNC gather ring per CTA: [warp][2 slots][UL][32] x 16 B
-template <int W, int V, int NR, typename TB, bool DYN>
-constexpr size_t seg_ring_bytes() {
-    return (size_t)(kBlock / 32) * 2 * seg_ul<W, V, NR, TB, false, DYN>() * 32 * 16;
-}
-
-// ASYNC: the B-row gathers go through asynchronous copies (cp.async, LDGSTS) into a
-// per-warp shared-memory ring of two batches, and the gathers of batch b+1 are issued
-// before batch b is processed (software pipelining without holding the next batch in
-// registers).  The replay of the workloads' own gather streams (profiles/r02) showed the
-// register-landing kernel at 0.60-0.64 of attainable on short rows and bf16: it has only
-// the current batch in flight while it settles rows.  2 CTAs/SM (shared memory).
 template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false,
-          bool DYN = false, bool ASYNC = false>
-__global__ void __launch_bounds__(kBlock, (ASYNC ? 2 : seg_min_blocks<W, V, TB, IT, DEEP>()))
+          bool DYN = false>
+__global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB, IT, DEEP>()))
 segment_kernel(const SegArgsT<IT> a) {
     using BV = BVec<TB, W>;
     using raw_t = typename BV::raw;
@@ -133,8 +121,6 @@ segment_kernel(const SegArgsT<IT> a) {
 
     __shared__ WarpStage stage[kWarps];
     __shared__ uint64_t bars[kWarps][2];
-    // ASYNC gather ring (dynamic shared memory): [warp][slot 0/1][UL][32 lanes] x 16 B
-    extern __shared__ __align__(16) uint4 seg_ring[];
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -429,40 +415,10 @@ segment_kernel(const SegArgsT<IT> a) {
             int q = ys - cb;
             q = q > 0 ? (q / U) * U : 0;
             const int qend = min(kCH, ye - cb);
-            // ASYNC: issue the copies of batch qq into ring slot sl (one commit group)
-            auto issue_async = [&](int qq, int sl) {
-                if constexpr (ASYNC) {
-                    static_assert(V == 1 && sizeof(raw_t) == 16, "async gathers: 16-B lanes");
-                    const int jj = cb + qq;
-                    uint4 *dst = seg_ring + (((size_t)warp * 2 + sl) * UL) * 32 + lane;
-#pragma unroll
-                    for (int i = 0; i < UL; ++i) {
-                        const int j = jj + i * NR + grp;
-                        const uint32_t c = (j >= ys && j < ye) ? (uint32_t)sc[qq + i * NR + grp] : 0u;
-                        cp_async16_l2(dst + i * 32, row_addr(bl[0], c, ldb_bytes), pol_last);
-                    }
-                    cp_async_commit();
-                }
-            };
-            int slot = 0;
-            if constexpr (ASYNC) {
-                if (q < qend) issue_async(q, 0);
-            }
             for (; q < qend; q += U) {
                 const int j0 = cb + q;
                 raw_t bv[UL][V];
                 const bool full = j0 >= ys && j0 + U <= ye;
-                if constexpr (ASYNC) {
-                    // next batch of this chunk in flight while this one is settled
-                    if (q + U < qend) issue_async(q + U, slot ^ 1);
-                    else cp_async_commit();                 // empty group: uniform waits
-                    cp_async_wait_group1();                 // this lane's copies of batch q
-                    const uint4 *src = seg_ring + (((size_t)warp * 2 + slot) * UL) * 32 + lane;
-#pragma unroll
-                    for (int i = 0; i < UL; ++i)
-                        bv[i][0] = *reinterpret_cast<const raw_t *>(src + i * 32);
-                    slot ^= 1;
-                } else {
                 // my non-zeros of this batch: u = i*NR + grp (i < UL).  Column indices
                 // and values are read as broadcast 16-B LDS of 4 consecutive entries
                 // (NR <= 4) and each lane selects its own; branch-free: outside the
@@ -512,8 +468,6 @@ segment_kernel(const SegArgsT<IT> a) {
                                                     row_addr(bl[s], cid[i], ldb_bytes)), pol);
                     }
                 }
-
-                }   // !ASYNC gathers
 
                 if (full && j0 + U <= rend) {
                     // fast path: U non-zeros of the current row, no checks
@@ -619,7 +573,7 @@ static bool dynamic_claims() {
 // concurrent first calls from several host threads only repeat the same query.
 template <typename KFn>
 static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic, KFn kdyn,
-                                     int *out, size_t dsm_st = 0, size_t dsm_dy = 0) {
+                                     int *out) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -639,22 +593,8 @@ static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic,
             e = cudaFuncSetAttribute(kdyn, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
         if (e != cudaSuccess) return e;
     }
-    if (dsm_st > 0 || dsm_dy > 0) {
-        // the ASYNC ring: two CTAs of ~97 KB need the maximum shared-memory carveout
-        e = cudaFuncSetAttribute(kstatic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm_st);
-        if (e == cudaSuccess)
-            e = cudaFuncSetAttribute(kdyn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)dsm_dy);
-        if (e == cudaSuccess && carve < 0)
-            e = cudaFuncSetAttribute(kstatic, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                     100);
-        if (e == cudaSuccess && carve < 0)
-            e = cudaFuncSetAttribute(kdyn, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-        if (e != cudaSuccess) return e;
-    }
     int bps = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kstatic, kBlock,
-                                                      dsm_st > dsm_dy ? dsm_st : dsm_dy);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kstatic, kBlock, 0);
     if (e != cudaSuccess) return e;
     if (bps < 1) bps = 1;
     if (dev >= 0 && dev < 64) cache[dev].store(bps, std::memory_order_relaxed);
@@ -662,18 +602,13 @@ static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic,
     return cudaSuccess;
 }
 
-template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false,
-          bool ASYNC = false>
+template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false>
 static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
-    auto kst = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false, ASYNC>;
-    auto kdy = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true, ASYNC>;
-    // ASYNC: the gather ring in dynamic shared memory (the same size for both variants
-    // is not guaranteed: each gets its own)
-    const size_t ring_st = ASYNC ? seg_ring_bytes<W, V, NR, TB, false>() : 0;
-    const size_t ring_dy = ASYNC ? seg_ring_bytes<W, V, NR, TB, true>() : 0;
+    auto kst = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, false>;
+    auto kdy = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>;
     static std::atomic<int> occ_cache[64];      // per instantiation, per device
     int blocks_per_sm = 0;
-    cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, &blocks_per_sm, ring_st, ring_dy);
+    cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, &blocks_per_sm);
     if (e != cudaSuccess) return e;
     const int64_t warps_per_block = kBlock / 32;
     int64_t need = (a.P + warps_per_block - 1) / warps_per_block;
@@ -700,7 +635,7 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = dim3(kBlock);
-    cfg.dynamicSmemBytes = dyn ? ring_dy : ring_st;
+    cfg.dynamicSmemBytes = 0;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -715,23 +650,13 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
 template <typename TB, int FIX, int W, typename IT>
 static cudaError_t dispatch_v(const SegArgsT<IT> &a, int V, int NR, cudaStream_t s) {
     if (V == 1) {
-        // 16-B lanes (fp32 x 4, bf16 x 8), int32 indices: the cp.async-pipelined gathers
-        constexpr bool kAsyncOk = W * (int)sizeof(TB) == 16 && sizeof(IT) == 4;
         switch (NR) {
-        case 1:
-            if constexpr (kAsyncOk)
-                if (a.async_gather) return launch_seg<W, 1, 1, TB, FIX, IT, false, true>(a, s);
-            return launch_seg<W, 1, 1, TB, FIX, IT>(a, s);
+        case 1: return launch_seg<W, 1, 1, TB, FIX, IT>(a, s);
         case 2:
-            if constexpr (kAsyncOk)
-                if (a.async_gather) return launch_seg<W, 1, 2, TB, FIX, IT, false, true>(a, s);
             if constexpr (W == 4 && sizeof(TB) == 4)
                 if (a.deep) return launch_seg<W, 1, 2, TB, FIX, IT, true>(a, s);
             return launch_seg<W, 1, 2, TB, FIX, IT>(a, s);
-        case 4:
-            if constexpr (kAsyncOk)
-                if (a.async_gather) return launch_seg<W, 1, 4, TB, FIX, IT, false, true>(a, s);
-            return launch_seg<W, 1, 4, TB, FIX, IT>(a, s);
+        case 4: return launch_seg<W, 1, 4, TB, FIX, IT>(a, s);
         case 8: return launch_seg<W, 1, 8, TB, FIX, IT>(a, s);
         case 16: return launch_seg<W, 1, 16, TB, FIX, IT>(a, s);
         case 32: return launch_seg<W, 1, 32, TB, FIX, IT>(a, s);

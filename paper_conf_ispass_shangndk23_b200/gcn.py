@@ -2,8 +2,10 @@
 
     out = A · ( relu( A · (X · W1) ) · W2 )           (A·(X·W) order P:282)
 
-The combination X·W is a plain dense GEMM (cuBLAS through torch.matmul -- a library GEMM,
-not on the SpMM hot path).  The aggregation A·B is MergePath-SpMM (libmpspmm), with the
+The combination X·W runs on the library's tcgen05 kernel (``mps_xw_bf16``, B in bf16
+straight into the gather layout; 1.2-3.3x cuBLAS on the GCN shapes, profiles/r02) wherever
+it applies (16 <= N <= 256, N % 16 == 0: ``combination="auto"``, the default), else as a
+plain cuBLAS GEMM (torch.matmul, fp32 B).  The aggregation A·B is MergePath-SpMM (libmpspmm), with the
 layer-1 ReLU fused into it (MPS_EPI_RELU: complete rows at the store, cut rows after
 their partial sums).  ``online=True`` recomputes the merge-path
 schedule on every inference (the paper's online setting) -- one partition per
@@ -20,11 +22,14 @@ from .api import CSR, Schedule, spmm, xw_bf16
 class GCN2:
     def __init__(self, A: CSR, W1: torch.Tensor, W2: torch.Tensor, online: bool = False,
                  b_dtype=torch.float32, fixup: str = "atomic", items_per_part: int = 0,
-                 min_parts: int = 0, combination: str = "cublas"):
+                 min_parts: int = 0, combination: str = "auto"):
         self.A, self.W1, self.W2 = A, W1, W2
         self.online, self.b_dtype, self.fixup = online, b_dtype, fixup
         # "tcgen05": X*W by the library's tensor-core kernel (mps_xw_bf16), B in bf16
         # straight into the gather layout (NEXT-3); "cublas": torch.matmul
+        if combination == "auto":
+            ok = all(16 <= w.shape[1] <= 256 and w.shape[1] % 16 == 0 for w in (W1, W2))
+            combination = "tcgen05" if ok else "cublas"
         self.combination = combination
         if combination == "tcgen05":
             self.b_dtype = torch.bfloat16

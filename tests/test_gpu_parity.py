@@ -348,7 +348,7 @@ def test_gcn2_layers_against_oracle(online):
     X = torch.randn(g.n, 128, generator=gen).cuda()
     W1 = (torch.randn(128, 64, generator=gen) / 11).cuda()
     W2 = (torch.randn(64, 16, generator=gen) / 8).cuda()
-    net = M.GCN2(A, W1, W2, online=online)
+    net = M.GCN2(A, W1, W2, online=online, combination="cublas")
     out = net(X)
     torch.cuda.synchronize()
     B1 = (X @ W1).cpu().numpy()
@@ -370,7 +370,8 @@ def test_gcn2_tcgen05_combination():
     X = torch.randn(g.n, 128, generator=gen).cuda()
     W1 = (torch.randn(128, 64, generator=gen) / 11).cuda()
     W2 = (torch.randn(64, 16, generator=gen) / 8).cuda()
-    net = M.GCN2(A, W1, W2, combination="tcgen05")
+    net = M.GCN2(A, W1, W2)                  # combination="auto" -> tcgen05 here
+    assert net.combination == "tcgen05"
     out = net(X)
     torch.cuda.synchronize()
     # layer 1: B1 = bf16(X) * bf16(W1) in fp32, rounded to bf16, checked vs fp64
