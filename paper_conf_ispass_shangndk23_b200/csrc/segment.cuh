@@ -68,6 +68,11 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP
 #define MPS_STATIC_ULCAP 4
 #endif
+// column indices / values of a batch: broadcast 16-B LDS of 4 entries + per-lane selects
+// when NR <= MPS_BCAST_NR, else one 4-B LDS per entry and lane
+#ifndef MPS_BCAST_NR
+#define MPS_BCAST_NR 4
+#endif
 #ifndef MPS_DYN_ULCAP
 #define MPS_DYN_ULCAP 0     // experiment: cap the dynamic instantiation's gathers per lane
 #endif
@@ -424,7 +429,7 @@ segment_kernel(const SegArgsT<IT> a) {
                 // (NR <= 4) and each lane selects its own; branch-free: outside the
                 // segment the column index is clamped to 0 (a harmless in-bounds row).
                 uint32_t cid[UL];
-                if constexpr (NR <= 4) {
+                if constexpr (NR <= MPS_BCAST_NR) {
 #pragma unroll
                     for (int t = 0; t < U / 4; ++t) {
                         const int4 c4 = *reinterpret_cast<const int4 *>(sc + q + 4 * t);
@@ -471,7 +476,7 @@ segment_kernel(const SegArgsT<IT> a) {
 
                 if (full && j0 + U <= rend) {
                     // fast path: U non-zeros of the current row, no checks
-                    if constexpr (NR <= 4) {
+                    if constexpr (NR <= MPS_BCAST_NR) {
 #pragma unroll
                         for (int t = 0; t < U / 4; ++t) {
                             const float4 v4 = *reinterpret_cast<const float4 *>(sv + q + 4 * t);
