@@ -69,9 +69,11 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #define MPS_STATIC_ULCAP 4
 #endif
 // column indices / values of a batch: broadcast 16-B LDS of 4 entries + per-lane selects
-// when NR <= MPS_BCAST_NR, else one 4-B LDS per entry and lane
+// when NR <= MPS_BCAST_NR, else one 4-B LDS per entry and lane.  Measured (r02o, same
+// box): per-lane LDS for NR >= 2 is 1-4% faster (R-MAT -2.6%, Reddit -0.9%, Pubmed -3%);
+// NR = 1 keeps the broadcast (compile-time picks, no selects).
 #ifndef MPS_BCAST_NR
-#define MPS_BCAST_NR 4
+#define MPS_BCAST_NR 1
 #endif
 #ifndef MPS_DYN_ULCAP
 #define MPS_DYN_ULCAP 0     // experiment: cap the dynamic instantiation's gathers per lane
