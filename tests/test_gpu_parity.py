@@ -580,6 +580,38 @@ def test_spmm_host_pipelined_chunks(monkeypatch, chunk, case):
         assert np.array_equal(Cs.numpy(), C.numpy())
 
 
+@pytest.mark.parametrize("serial", [False, True])
+def test_spmm_host_strided_buffers_keep_padding(monkeypatch, serial):
+    """with ldc > K (a strided C_host view) the host calls write only the K
+    valid columns of each row -- the padding of the caller's host matrix keeps its
+    sentinel -- and with ldb > K they read only the K valid columns of B_host (the
+    B_host view ends before the padding of its last row)."""
+    g = G.workload("pubmed")
+    A = dev(g)
+    K, ldb, ldc = 64, 72, 80
+    Bfull = np.full((g.n, ldb), np.nan, np.float32)
+    Bfull[:, :K] = G.dense_int(g.n, K, seed=5)
+    ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, Bfull[:, :K], want_bound=False)
+    pin = lambda a: torch.from_numpy(a).pin_memory()
+    Bh = pin(Bfull)[:, :K]                          # stride(0) = ldb > K
+    if serial:
+        monkeypatch.setenv("MPS_HOST_SERIAL", "1")
+    for call in ("host", "host_dense"):
+        Cbuf = torch.full((g.m, ldc), -7.0, dtype=torch.float32).pin_memory()
+        Ch = Cbuf[:, :K]                            # stride(0) = ldc > K
+        if call == "host":
+            M.spmm_host(pin(g.row_ptr), pin(g.col_idx), pin(g.val), g.n, Bh, C_host=Ch)
+        else:
+            M.spmm_host_dense(A, Bh, C_host=Ch)
+        out = Cbuf.numpy()
+        assert np.all(out[:, K:] == -7.0), call         # padding untouched
+        # integer-valued B with GCN-normalised A: within the north-star tolerance
+        bnd = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, np.abs(Bfull[:, :K]),
+                             want_bound=False)
+        r = O.check(out[:, :K], ref, bnd)
+        assert r["ok"], (call, r)
+
+
 @pytest.mark.parametrize("fixup", ["atomic", "carry"])
 def test_spmm_host_dense_graph_resident(fixup):
     g = G.workload("pubmed")
