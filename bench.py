@@ -602,8 +602,12 @@ def main():
             cg.replay()
         stream = torch.cuda.current_stream(dev)
 
-    inner_events = not (args.cuda_graph and world == 1) and not (
-        world == 1 and online.path == L.MPS_PATH_SMALL_FUSED)
+    small_path = world == 1 and online.path == L.MPS_PATH_SMALL_FUSED
+    if world == 1:
+        launches_per_step = online.launches(l2)    # the path is resolved by the warm-up
+    path_desc = ("small_fused (1 kernel + carry reduction)" if small_path else
+                 "partition+segments") if world == 1 else "sharded"
+    inner_events = not (args.cuda_graph and world == 1) and not small_path
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
             torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
            for _ in range(args.steps)]
@@ -743,7 +747,7 @@ def main():
     # column pattern produces; roofline.peak is the algorithmic byte rate at that time.
     row_bytes = tile_cols * b_elt
     if world == 1 and not args.no_l2_probe and row_bytes in (64, 128, 256, 512) \
-            and online.path != L.MPS_PATH_SMALL_FUSED:
+            and not small_path:
         try:
             import __graft_entry__
             gr = ctypes.CDLL(__graft_entry__.build_gather_replay())
@@ -914,9 +918,7 @@ def main():
             "config": {
                 "workload": "%s-k%d" % (name, K), "graph": g.name, "n": g.m, "nnz": g.nnz,
                 "K": K, "b_dtype": args.dtype, "fixup": args.fixup,
-                "path": (("small_fused (1 kernel + carry reduction)"
-                          if online.path == L.MPS_PATH_SMALL_FUSED else
-                          "partition+segments") if world == 1 else "sharded"),
+                "path": path_desc,
                 "num_parts": P, "items_per_part": Lp, "mode": "online (partition every step)",
                 "timing": "CUDA events around each step on the launching stream, every step "
                           "synchronised (the cuSPARSE reference's protocol); value = mean",

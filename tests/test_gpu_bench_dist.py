@@ -38,3 +38,26 @@ def test_bench_two_ranks(tails):
     assert d["n_gpus"] == 2 and d["steps"] == 3 and d["value"] > 0
     assert d["config"]["tail_exchange"] == tails
     assert d["parity"]["ok"] and d["parity"]["all_ranks_ok"]
+
+
+@pytest.mark.parametrize("wl,K,extra", [("pubmed", 64, []), ("rmat", 64, []),
+                                        ("cora", 16, ["--cuda-graph"])])
+def test_bench_single_gpu_all_legs(wl, K, extra):
+    """The N = 1 bench line with every leg on (e2e through the host-buffer ABI, the CPU
+    baseline, cuSPARSE, L2 probe, gather replay, parity check): one JSON line carrying
+    the contract's keys."""
+    cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--workload", wl, "--K", str(K),
+           "--steps", "3", "--warmup", "3", "--e2e-steps", "1", "--cpu-seconds", "1"] + extra
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    lines = [json.loads(ln) for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = lines[0]
+    for key in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step",
+                "higher_is_better", "scaling", "vs_baseline", "dtype", "data", "config",
+                "roofline", "cpu_baseline", "e2e", "gpu_launches", "clocks", "parity"):
+        assert key in d, key
+    assert d["value"] > 0 and d["gpu_launches"] > 0 and d["parity"]["ok"]
+    assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert {"bound", "achieved", "peak", "unit", "frac"} <= set(d["roofline"])
