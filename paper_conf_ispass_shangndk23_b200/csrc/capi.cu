@@ -236,12 +236,6 @@ int64_t host_diag_x(const IT *rp, int64_t m, int64_t nnz, int64_t d) {
     return lo - 1;
 }
 
-// rows of B a schedule gathers from: every column of A may be referenced, so the
-// conservative count is the number of B rows, which the caller does not pass here --
-// a.n_b_rows (set by the entry points) carries it
-template <typename IT>
-int64_t base_rows_of(const mps::SegArgsT<IT> &a) { return a.n_b_rows; }
-
 // Run a3 (+ a4 carry reduction) over all column tiles for a ready schedule.
 // claims: the per-tile claim counters (workspace; NULL: static segment assignment);
 // claims_zeroed: a kernel earlier on the stream already zeroed them, else they are
@@ -278,17 +272,6 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
         int V, NR;
         tile_geometry(kt, v.W, &V, &NR);
         a.deep = v.deep && kt == 64 ? 1 : 0;
-        // L2 prefetch of the next batch's B rows where the tile's B slice exceeds half the
-        // L2 (its gathers miss); MPS_L2PF=0/1 overrides.  Needs 16-B rows.
-        static const int l2pf_env = [] {
-            const char *e = getenv("MPS_L2PF");
-            return e ? atoi(e) : -1;
-        }();
-        a.row_bytes = (uint32_t)kt * (uint32_t)eb;
-        const bool b_beyond_l2 = (double)base_rows_of(base) * kt * eb > 0.5 * (double)l2_bytes();
-        a.l2_prefetch = ((l2pf_env == 1 || (l2pf_env < 0 && b_beyond_l2)) &&
-                         a.row_bytes % 16 == 0 && (((uintptr_t)a.B) & 15u) == 0 &&
-                         (a.ldb * eb) % 16 == 0) ? 1 : 0;
         mps::SegArgsT<IT> seg_only = a;
         seg_only.mail.on = 0;
         MPS_CUDA(mps::launch_segments(fix == mps::FIX_CARRY ? seg_only : a, dt, v.W, V, NR, fix,
@@ -501,7 +484,6 @@ mps_status segments_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t l
     a.tail_row = -1;
     a.tail = nullptr;
     a.nnz_end = A->nnz;
-    a.n_b_rows = A->n;
     a.hot = hot_bitmap;
     a.relu = relu;
     a.wstat = wstat;
@@ -772,7 +754,6 @@ mps_status online_ex_impl(const CSR *A, const void *B, int32_t b_dtype, int64_t 
     a.tail_row = -1;
     a.tail = nullptr;
     a.nnz_end = A->nnz;
-    a.n_b_rows = A->n;
     a.hot = bitmap;
     a.relu = epilogue == MPS_EPI_RELU;
     return run_segments(a, b_dtype, K, v, fix, rec, claims, nz > 0, s);
@@ -1128,7 +1109,6 @@ static mps_status host_pipelined(const mps_csr *A_host, const void *B_host, int3
             a.tail_row = -1;
             a.tail = nullptr;
             a.nnz_end = nnz;
-            a.n_b_rows = A_host->n;
             a.hot = nullptr;
             a.relu = 0;
             // static segment assignment: the chunks' launches would each need their
@@ -1582,7 +1562,6 @@ static mps_status shard_impl(const CSR *A, const void *B, int32_t b_dtype, int64
     a.tail_row = trow;
     a.tail = tail_out;
     a.nnz_end = (int64_t)Y[rank + 1];
-    a.n_b_rows = A->n;
     a.mail = mail;
     return run_segments(a, b_dtype, K, v, fix, rec, claims, nz > 0, s);
 }

@@ -78,9 +78,6 @@ struct SegArgsT {
     unsigned *claim;     // dynamic segment claims: this column tile's counter in the caller's
                          // workspace, zero when the kernel starts (NULL: static assignment)
     int32_t deep;        // 1: deep-gather instantiation (fp32, 64-column tile, DRAM-bound B)
-    int32_t l2_prefetch; // 1: bulk-prefetch the next batch's B rows into L2 (B beyond L2)
-    uint32_t row_bytes;  // bytes of one B row of this column tile (multiple of 16)
-    int64_t n_b_rows;    // rows of B (columns of A), for the launch-time L2 decisions
     unsigned long long *wstat;  // Fig. 5 counters of what the kernel wrote (NULL: off):
                                 // [0] partial-row updates (atomic / carry record),
                                 // [1] empty partial start pieces whose add was elided,
@@ -371,11 +368,6 @@ __device__ __forceinline__ void cp_async8(void *dst_smem, const void *src) {
 __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.wait_all;" ::: "memory");
 }
-// bulk prefetch of `bytes` (multiple of 16, 16-B aligned) into L2; no completion tracking
-__device__ __forceinline__ void prefetch_l2_bulk(const void *p, uint32_t bytes) {
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(bytes) : "memory");
-}
-
 // global -> shared bulk copy of `bytes` (multiple of 16, both addresses 16-B aligned),
 // completion counted on `bar`; L2 evict_first (streamed once).
 __device__ __forceinline__ void tma_load_1d(void *dst, const void *src, uint32_t bytes,

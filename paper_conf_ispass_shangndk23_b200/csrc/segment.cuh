@@ -426,15 +426,6 @@ segment_kernel(const SegArgsT<IT> a) {
                 const int j0 = cb + q;
                 raw_t bv[UL][V];
                 const bool full = j0 >= ys && j0 + U <= ye;
-                // B rows of the NEXT batch of this chunk into L2 (bulk prefetch, no
-                // registers held): where B does not fit in L2 the gathers of that batch
-                // then wait for an L2 hit instead of a DRAM miss
-                if (a.l2_prefetch && q + U < qend && lane < U) {
-                    const int jn = j0 + U + lane;
-                    if (jn < ye)
-                        prefetch_l2_bulk(row_addr(Bc, (uint32_t)sc[q + U + lane], ldb_bytes),
-                                         a.row_bytes);
-                }
                 // my non-zeros of this batch: u = i*NR + grp (i < UL).  Column indices
                 // and values are read as broadcast 16-B LDS of 4 consecutive entries
                 // (NR <= 4) and each lane selects its own; branch-free: outside the
