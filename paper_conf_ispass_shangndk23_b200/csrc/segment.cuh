@@ -85,11 +85,6 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 // 1 = step by step (one warp instruction's NR non-zeros at a time).  Measured on B200
 // (profiles/r02/slow_steps.md): the step form is 1.6x slower on R-MAT and 2.3x on
 // products (register spills and serialised per-step control flow), so 0 stays.
-// slow-path passes skip the batch entries outside the current row's range (uniform
-// branches) -- measured in profiles/r02/pass_skip.md
-#ifndef MPS_PASS_SKIP
-#define MPS_PASS_SKIP 0
-#endif
 #ifndef MPS_SLOW_STEPS
 #define MPS_SLOW_STEPS 0
 #endif
@@ -544,14 +539,6 @@ segment_kernel(const SegArgsT<IT> a) {
                         const int lim = rend < jend ? rend : jend;  // row r's part: [jc, lim)
 #pragma unroll
                         for (int i = 0; i < UL; ++i) {
-#if MPS_PASS_SKIP
-                            // warp-uniform: entries (warp instructions) wholly outside
-                            // [jc, lim) are skipped, so the passes of a batch together
-                            // touch ~UL + (row ends) entries instead of (passes) x UL
-                            const int jb = j0 + i * NR;
-                            if (jb >= lim) break;
-                            if (jb + NR <= jc) continue;
-#endif
                             const int j = j0 + i * NR + grp;
                             if (j >= jc && j < lim) fma_row(vl[i], bv[i]);
                         }
