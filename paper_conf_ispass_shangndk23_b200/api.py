@@ -132,14 +132,15 @@ def _keep(t, stream):
 EPILOGUE = {"none": L.MPS_EPI_NONE, "relu": L.MPS_EPI_RELU}
 
 
-def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomic",
+def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="auto",
          items_per_part=0, min_parts=0, out: torch.Tensor | None = None, stream=None,
          epilogue="none"):
     """C = A * B (row-wise product) by MergePath-SpMM.
 
     With ``schedule`` the offline path (mps_spmm) runs; otherwise the online path
-    (mps_spmm_online: plan + partition + SpMM).  B: (n, K) float32/bfloat16 on A's
-    device, rows may be padded (B.stride(0) = ldb >= K).  Returns C (m, K) float32."""
+    (mps_spmm_online: plan + partition + SpMM; with the default fixup "auto" small graphs
+    take the one-launch small-graph path).  B: (n, K) float32/bfloat16 on A's device,
+    rows may be padded (B.stride(0) = ldb >= K).  Returns C (m, K) float32."""
     assert B.dim() == 2 and B.stride(1) == 1 and B.device == A.device
     K = B.shape[1]
     dt = _dtype_code(B)
@@ -184,14 +185,15 @@ def spmm(A: CSR, B: torch.Tensor, schedule: Schedule | None = None, fixup="atomi
 
 
 class CapturedSpMM:
-    """The online path (mps_spmm_online: partition + zeroing + segment kernel) captured
-    once in a CUDA graph for fixed A, B and C buffers, then replayed.  Replay removes
+    """The online path (mps_spmm_online: partition + zeroing + segment kernel, or the
+    one-launch small-graph path) captured once in a CUDA graph for fixed A, B and C
+    buffers, then replayed.  Replay removes
     the per-call host launch overhead that dominates small graphs (Cora, Pubmed), and
     keeps the paper's online setting -- the schedule is recomputed on every call
     (P:151).  Update B / A values in place between replays."""
 
     def __init__(self, A: CSR, B: torch.Tensor, out: torch.Tensor | None = None,
-                 fixup="atomic", items_per_part=0, min_parts=0):
+                 fixup="auto", items_per_part=0, min_parts=0):
         self.A, self.B = A, B
         self.K = B.shape[1]
         self.C = torch.empty((A.m, self.K), dtype=torch.float32, device=A.device) \

@@ -121,7 +121,9 @@ def test_full_matrix_f32(name, K):
     for _ in range(2):                  # twice: the claim counters are reused across calls
         st(Bt)
     outs["bench_path_atomic"] = st.C
-    outs["online_atomic"] = M.spmm(A, Bt, out=torch.full((g.m, K), float("nan"), device="cuda"))
+    outs["online_atomic"] = M.spmm(A, Bt, fixup="atomic",
+                                   out=torch.full((g.m, K), float("nan"), device="cuda"))
+    outs["online_auto"] = M.spmm(A, Bt, out=torch.full((g.m, K), float("nan"), device="cuda"))
     outs["online_carry"] = M.spmm(A, Bt, fixup="carry",
                                   out=torch.full((g.m, K), float("nan"), device="cuda"))
     torch.cuda.synchronize()
