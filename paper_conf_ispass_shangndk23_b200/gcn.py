@@ -14,6 +14,8 @@ call (the offline default).
 """
 from __future__ import annotations
 
+import ctypes
+
 import torch
 
 from .api import CSR, Schedule, spmm, xw_bf16
@@ -21,7 +23,7 @@ from .api import CSR, Schedule, spmm, xw_bf16
 
 class GCN2:
     def __init__(self, A: CSR, W1: torch.Tensor, W2: torch.Tensor, online: bool = False,
-                 b_dtype=torch.float32, fixup: str = "atomic", items_per_part: int = 0,
+                 b_dtype=torch.float32, fixup: str = "auto", items_per_part: int = 0,
                  min_parts: int = 0, combination: str = "auto"):
         self.A, self.W1, self.W2 = A, W1, W2
         self.online, self.b_dtype, self.fixup = online, b_dtype, fixup
@@ -39,10 +41,31 @@ class GCN2:
         self.H = torch.empty((A.m, W1.shape[1]), dtype=torch.float32, device=A.device)
         self.out = torch.empty((A.m, W2.shape[1]), dtype=torch.float32, device=A.device)
         # the default plan depends on the graph only, so one schedule serves both layers
-        self.schedule = None if online else Schedule.build(A, W1.shape[1], b_dtype,
+        self.schedule = None if online else Schedule.build(A, W1.shape[1], self.b_dtype,
                                                            items_per_part, min_parts)
+        # online on a small graph: each aggregation is one mps_spmm_online call on the
+        # one-launch small-graph path (it computes its own schedule inside the kernel)
+        self.fused_online = False
+        if online and not A.wide:
+            from . import _lib as L
+            path = ctypes.c_int32()
+            a = A.struct()
+            ok = True
+            for w in (W1, W2):
+                L.mps_spmm_online_path(ctypes.byref(a), None,
+                                       L.MPS_DT_BF16 if self.b_dtype == torch.bfloat16
+                                       else L.MPS_DT_F32, w.shape[1], w.shape[1], None,
+                                       w.shape[1], items_per_part, min_parts,
+                                       L.MPS_FIXUP_AUTO if fixup == "auto" else
+                                       (L.MPS_FIXUP_CARRY if fixup == "carry" else
+                                        L.MPS_FIXUP_ATOMIC), ctypes.byref(path))
+                ok = ok and path.value == L.MPS_PATH_SMALL_FUSED
+            self.fused_online = ok
 
     def _aggregate(self, B, out, epilogue):
+        if self.fused_online:
+            return spmm(self.A, B.to(self.b_dtype), fixup=self.fixup, items_per_part=self.ipp,
+                        min_parts=self.minp, out=out, epilogue=epilogue)
         return spmm(self.A, B.to(self.b_dtype), schedule=self.schedule, fixup=self.fixup,
                     items_per_part=self.ipp, min_parts=self.minp, out=out, epilogue=epilogue)
 
@@ -56,7 +79,7 @@ class GCN2:
                                "relu")
 
     def __call__(self, X: torch.Tensor) -> torch.Tensor:
-        if self.online:
+        if self.online and not self.fused_online:
             # online setting: the schedule is recomputed for every inference --
             # once, since the default plan depends on the graph only, for both layers
             self.schedule = Schedule.build(self.A, self.W1.shape[1], self.b_dtype, self.ipp,

@@ -34,9 +34,12 @@ def main():
         W1 = (torch.randn(F, H, generator=gen) / F ** 0.5).cuda()
         W2 = (torch.randn(H, C, generator=gen) / H ** 0.5).cuda()
         row = {"workload": wl, "n": g.m, "nnz": g.nnz, "F": F, "H": H, "C": C}
-        for mode in ("offline", "online", "offline_tcgen05"):
-            net = M.GCN2(A, W1, W2, online=(mode == "online"),
-                         combination="tcgen05" if "tcgen05" in mode else "cublas")
+        # default GCN2: tcgen05 combination (bf16 B) where it applies; online on a small
+        # graph = the one-launch small-graph path per aggregation
+        for mode in ("offline", "online", "offline_cublas", "online_cublas"):
+            net = M.GCN2(A, W1, W2, online=mode.startswith("online"),
+                         combination="cublas" if "cublas" in mode else "auto")
+            row[mode + "_fused_online"] = bool(net.fused_online)
             row[mode + "_ms"] = time_it(lambda: net(X))
             g_ = torch.cuda.CUDAGraph()
             net(X); torch.cuda.synchronize()
@@ -45,10 +48,12 @@ def main():
             row[mode + "_graph_ms"] = time_it(g_.replay)
         row["online_overhead_pct"] = 100 * (row["online_ms"] / row["offline_ms"] - 1)
         row["online_overhead_graph_pct"] = 100 * (row["online_graph_ms"] / row["offline_graph_ms"] - 1)
+        row["online_overhead_cublas_graph_pct"] = 100 * (row["online_cublas_graph_ms"] /
+                                                         row["offline_cublas_graph_ms"] - 1)
         print(json.dumps(row), flush=True)
         res.append(row)
-    ov = [max(r["online_overhead_graph_pct"], 1e-3) for r in res]
-    print(json.dumps({"geomean_online_overhead_graph_pct": float(np.exp(np.mean(np.log(ov))))}))
+    ratio = [r["online_graph_ms"] / r["offline_graph_ms"] for r in res]
+    print(json.dumps({"geomean_online_over_offline_graph": float(np.exp(np.mean(np.log(ratio))))}))
 
 
 if __name__ == "__main__":
