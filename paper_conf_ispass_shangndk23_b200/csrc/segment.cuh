@@ -81,13 +81,6 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP_MINNR
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
-// slow path of the segment walk: 0 = one pass over the whole batch per row touching it;
-// 1 = step by step (one warp instruction's NR non-zeros at a time).  Measured on B200
-// (profiles/r02/slow_steps.md): the step form is 1.6x slower on R-MAT and 2.3x on
-// products (register spills and serialised per-step control flow), so 0 stays.
-#ifndef MPS_SLOW_STEPS
-#define MPS_SLOW_STEPS 0
-#endif
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
 #endif
@@ -493,40 +486,6 @@ segment_kernel(const SegArgsT<IT> a) {
                     }
                 } else {
                     // slow path: the batch crosses row ends (or the segment's edges).
-#if MPS_SLOW_STEPS
-                    // Step by step (step i = the NR non-zeros j0 + i*NR .. + NR-1 of one
-                    // warp instruction): rows that end before the step are settled, then
-                    // a step inside row r is one predicated FMA; only a step that a row
-                    // end cuts takes one pass per row.  Cost ~ UL + (row ends) FMA
-                    // passes, not (1 + row ends) * UL as with whole-batch passes -- the
-                    // difference on short-row graphs (R-MAT: median row length 1).
-                    float vl[UL];
-#pragma unroll
-                    for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
-                    const int lo = j0 > ys ? j0 : ys;            // the batch's part of the
-                    const int hi = (j0 + U < ye) ? j0 + U : ye;  // segment: [lo, hi)
-#pragma unroll
-                    for (int i = 0; i < UL; ++i) {
-                        const int jb = j0 + i * NR;
-                        const int sb = jb > lo ? jb : lo;
-                        const int se = (jb + NR < hi) ? jb + NR : hi;
-                        if (sb < se) {                           // warp-uniform
-                            while (sb >= rend) finish_row();     // rows ending before the step
-                            const int j = jb + grp;
-                            if (se <= rend) {
-                                if (j >= sb && j < se) fma_row(vl[i], bv[i]);
-                            } else {                             // a row end inside the step
-                                int c = sb;
-                                while (c < se) {
-                                    while (c >= rend) finish_row();
-                                    const int lim = rend < se ? rend : se;
-                                    if (j >= c && j < lim) fma_row(vl[i], bv[i]);
-                                    c = lim;
-                                }
-                            }
-                        }
-                    }
-#else
                     // One pass per row intersecting the batch: predicated FMAs for the
                     // non-zeros of the current row, then settle the row.
                     float vl[UL];
@@ -544,7 +503,6 @@ segment_kernel(const SegArgsT<IT> a) {
                         }
                         jc = lim;
                     }
-#endif
                 }
             }
             ++ccount;
