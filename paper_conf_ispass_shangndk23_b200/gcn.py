@@ -30,8 +30,11 @@ class GCN2:
         # "tcgen05": X*W by the library's tensor-core kernel (mps_xw_bf16), B in bf16
         # straight into the gather layout (NEXT-3); "cublas": torch.matmul
         if combination == "auto":
+            # tcgen05 where the kernel applies, except tiny graphs: on Cora (2,708 rows)
+            # cuBLAS's X*W is 4 us faster per inference, from Pubmed (19,717) up tcgen05
+            # wins (profiles/r02/gcn_online_offline.md)
             ok = all(16 <= w.shape[1] <= 256 and w.shape[1] % 16 == 0 for w in (W1, W2))
-            combination = "tcgen05" if ok else "cublas"
+            combination = "tcgen05" if ok and A.m >= 8192 else "cublas"
         self.combination = combination
         if combination == "tcgen05":
             self.b_dtype = torch.bfloat16
