@@ -81,6 +81,9 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP_MINNR
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
+#ifndef MPS_SLOW_PARTS
+#define MPS_SLOW_PARTS 1
+#endif
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
 #endif
@@ -491,17 +494,28 @@ segment_kernel(const SegArgsT<IT> a) {
                     float vl[UL];
 #pragma unroll
                     for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
+                    // The batch is settled in SP parts of UL/SP entries each; a part's
+                    // passes predicate only its own entries, so a row end costs UL/SP
+                    // FMA groups instead of UL (MPS_SLOW_PARTS, measured in
+                    // profiles/r02/slow_steps.md)
+                    constexpr int SP = (MPS_SLOW_PARTS >= 1 && UL % MPS_SLOW_PARTS == 0)
+                                           ? MPS_SLOW_PARTS : 1;
+                    constexpr int ULP = UL / SP;
                     int jc = j0 > ys ? j0 : ys;                  // next non-zero to consume
-                    const int jend = (j0 + U < ye) ? j0 + U : ye;
-                    while (jc < jend) {
-                        while (jc >= rend) finish_row();          // rows ending before jc
-                        const int lim = rend < jend ? rend : jend;  // row r's part: [jc, lim)
 #pragma unroll
-                        for (int i = 0; i < UL; ++i) {
-                            const int j = j0 + i * NR + grp;
-                            if (j >= jc && j < lim) fma_row(vl[i], bv[i]);
+                    for (int h = 0; h < SP; ++h) {
+                        const int pe = j0 + (h + 1) * ULP * NR;
+                        const int jend = pe < ye ? pe : ye;
+                        while (jc < jend) {
+                            while (jc >= rend) finish_row();      // rows ending before jc
+                            const int lim = rend < jend ? rend : jend;  // row r's part
+#pragma unroll
+                            for (int i = h * ULP; i < (h + 1) * ULP; ++i) {
+                                const int j = j0 + i * NR + grp;
+                                if (j >= jc && j < lim) fma_row(vl[i], bv[i]);
+                            }
+                            jc = lim;
                         }
-                        jc = lim;
                     }
                 }
             }
