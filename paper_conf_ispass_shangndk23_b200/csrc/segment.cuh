@@ -82,7 +82,7 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
 #ifndef MPS_SLOW_PARTS
-#define MPS_SLOW_PARTS 1
+#define MPS_SLOW_PARTS 0     // 0: the measured rule below (2 parts for >= 32-non-zero batches)
 #endif
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
@@ -498,8 +498,10 @@ segment_kernel(const SegArgsT<IT> a) {
                     // passes predicate only its own entries, so a row end costs UL/SP
                     // FMA groups instead of UL (MPS_SLOW_PARTS, measured in
                     // profiles/r02/slow_steps.md)
-                    constexpr int SP = (MPS_SLOW_PARTS >= 1 && UL % MPS_SLOW_PARTS == 0)
-                                           ? MPS_SLOW_PARTS : 1;
+                    // (default: two parts for batches of >= 32 non-zeros -- bf16 K=64 /
+                    // fp32 K=32 -- where they measured 4-6% faster; one part otherwise)
+                    constexpr int SP0 = MPS_SLOW_PARTS > 0 ? MPS_SLOW_PARTS : (U >= 32 ? 2 : 1);
+                    constexpr int SP = (UL % SP0 == 0) ? SP0 : 1;
                     constexpr int ULP = UL / SP;
                     int jc = j0 > ys ? j0 : ys;                  // next non-zero to consume
 #pragma unroll
