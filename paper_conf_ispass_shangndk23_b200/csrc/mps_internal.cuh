@@ -176,6 +176,12 @@ template <bool ON>
 __device__ __forceinline__ void count_write_if(unsigned long long *wstat, int lane, int k) {
     if constexpr (ON) count_write(wstat, lane, k);
 }
+template <bool ON>
+__device__ __forceinline__ void count_write_n_if(unsigned long long *wstat, int lane, int k,
+                                                 int n) {
+    if constexpr (ON)
+        if (wstat != nullptr && lane == 0 && n > 0) atomicAdd(wstat + k, (unsigned long long)n);
+}
 __device__ __forceinline__ int ld_stream_i32(const int32_t *p) {
     int v;
     asm volatile("ld.global.cs.s32 %0, [%1];" : "=r"(v) : "l"(p));

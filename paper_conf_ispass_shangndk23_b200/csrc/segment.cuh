@@ -81,6 +81,9 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP_MINNR
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
+#ifndef MPS_EMPTY_RUNS
+#define MPS_EMPTY_RUNS 0     // experiment: batched zero stores for runs of empty rows
+#endif
 #ifndef MPS_SLOW_PARTS
 #define MPS_SLOW_PARTS 0     // 0: the measured rule below (2 parts for >= 32-non-zero batches)
 #endif
@@ -405,6 +408,44 @@ segment_kernel(const SegArgsT<IT> a) {
             }
         };
 
+#if MPS_EMPTY_RUNS
+        // A run of empty rows starting at r (rp[r+1] == rbeg ...) is settled with one
+        // zero store per NR rows -- no butterfly, no per-row walk (nothing accumulated;
+        // R-MAT: 48% of its rows are empty).  Rows stay below xe (their end items lie in
+        // this segment); the window lanes give the run length by one ballot.
+        auto zero_empty_run = [&]() {
+            while (r < xe && rend == rbeg) {
+                int idx = r + 1 - wb;
+                const unsigned eq = __ballot_sync(0xffffffffu, win == rbeg);
+                const unsigned run = ~(eq >> idx);
+                int k = run ? __ffs(run) - 1 : 32 - idx;
+                k = k < xe - r ? k : xe - r;
+                {   // every lane group stores its own rows of the run
+                    for (int t = grp; t < k; t += NR) {
+                        float *dst = a.C + ((int64_t)(r + t) - a.row_base) * a.ldc;
+#pragma unroll
+                        for (int s = 0; s < V; ++s)
+                            if (act[s]) {
+                                float z[W];
+#pragma unroll
+                                for (int w = 0; w < W; ++w) z[w] = 0.f;
+                                CVec<W>::store(dst + cofs[s], z);
+                            }
+                    }
+                }
+                count_write_n_if<!DYN>(a.wstat, lane, 2, k);
+                r += k;
+                idx = r + 1 - wb;
+                if (idx >= 32) {
+                    wb = r;
+                    win = rel((wb + lane <= m) ? __ldg(rp + wb + lane) : kInf);
+                    idx = 1;
+                }
+                rend = __shfl_sync(0xffffffffu, win, idx);      // rbeg is unchanged
+            }
+        };
+#endif
+
         for (int k = 0; k < nch; ++k) {
             if (!direct) {
                 mbar_wait(&bars[warp][ccount & 1u], (ccount >> 1) & 1u);
@@ -509,7 +550,12 @@ segment_kernel(const SegArgsT<IT> a) {
                         const int pe = j0 + (h + 1) * ULP * NR;
                         const int jend = pe < ye ? pe : ye;
                         while (jc < jend) {
-                            while (jc >= rend) finish_row();      // rows ending before jc
+                            while (jc >= rend) {                  // rows ending before jc
+                                finish_row();
+#if MPS_EMPTY_RUNS
+                                zero_empty_run();
+#endif
+                            }
                             const int lim = rend < jend ? rend : jend;  // row r's part
 #pragma unroll
                             for (int i = h * ULP; i < (h + 1) * ULP; ++i) {
@@ -524,7 +570,12 @@ segment_kernel(const SegArgsT<IT> a) {
             ++ccount;
         }
         // rows whose end item lies in this segment after its last non-zero
-        while (r < xe) finish_row();
+        while (r < xe) {
+            finish_row();
+#if MPS_EMPTY_RUNS
+            zero_empty_run();
+#endif
+        }
 
         // r == xe: the segment's non-zeros of row xe, if any (lines 3-5 / 11-13)
         if (xe < m && ye > rbeg) {
