@@ -81,8 +81,10 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_STATIC_ULCAP_MINNR
 #define MPS_STATIC_ULCAP_MINNR 2
 #endif
+// batched zero stores for runs of empty rows: -1 = the measured rule (fp32 B, not the
+// deep-gather kernel: R-MAT -2.3%, Reddit neutral; bf16 Reddit +2%, products +1.5%), 0/1
 #ifndef MPS_EMPTY_RUNS
-#define MPS_EMPTY_RUNS 0     // experiment: batched zero stores for runs of empty rows
+#define MPS_EMPTY_RUNS -1
 #endif
 #ifndef MPS_SLOW_PARTS
 #define MPS_SLOW_PARTS 0     // 0: the measured rule below (2 parts for >= 32-non-zero batches)
@@ -408,12 +410,14 @@ segment_kernel(const SegArgsT<IT> a) {
             }
         };
 
-#if MPS_EMPTY_RUNS
+        constexpr bool kEmptyRuns = MPS_EMPTY_RUNS >= 0 ? (MPS_EMPTY_RUNS != 0)
+                                                        : (sizeof(TB) == 4 && !DEEP);
         // A run of empty rows starting at r (rp[r+1] == rbeg ...) is settled with one
         // zero store per NR rows -- no butterfly, no per-row walk (nothing accumulated;
         // R-MAT: 48% of its rows are empty).  Rows stay below xe (their end items lie in
         // this segment); the window lanes give the run length by one ballot.
         auto zero_empty_run = [&]() {
+            if constexpr (!kEmptyRuns) return;
             while (r < xe && rend == rbeg) {
                 int idx = r + 1 - wb;
                 const unsigned eq = __ballot_sync(0xffffffffu, win == rbeg);
@@ -444,7 +448,6 @@ segment_kernel(const SegArgsT<IT> a) {
                 rend = __shfl_sync(0xffffffffu, win, idx);      // rbeg is unchanged
             }
         };
-#endif
 
         for (int k = 0; k < nch; ++k) {
             if (!direct) {
@@ -552,9 +555,7 @@ segment_kernel(const SegArgsT<IT> a) {
                         while (jc < jend) {
                             while (jc >= rend) {                  // rows ending before jc
                                 finish_row();
-#if MPS_EMPTY_RUNS
                                 zero_empty_run();
-#endif
                             }
                             const int lim = rend < jend ? rend : jend;  // row r's part
 #pragma unroll
@@ -572,9 +573,7 @@ segment_kernel(const SegArgsT<IT> a) {
         // rows whose end item lies in this segment after its last non-zero
         while (r < xe) {
             finish_row();
-#if MPS_EMPTY_RUNS
             zero_empty_run();
-#endif
         }
 
         // r == xe: the segment's non-zeros of row xe, if any (lines 3-5 / 11-13)
