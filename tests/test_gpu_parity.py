@@ -739,5 +739,8 @@ def test_bench_cuda_graph_replays_the_step(wl, K):
         assert r.returncode == 0, r.stderr[-2000:]
         lines[mode] = json.loads([ln for ln in r.stdout.splitlines() if ln.startswith("{")][-1])
     assert lines["graph"]["config"]["cuda_graph"] is True
-    # the eager step's segment kernel alone bounds the graph replay from below
-    assert lines["graph"]["ms_per_step"] >= 0.5 * lines["eager"]["segment_ms"]
+    # the eager step's segment kernel alone bounds the graph replay from below (its
+    # fastest eager step: on tiny graphs one slow step inflates the eager mean)
+    eager = lines["eager"]
+    floor = min(eager["segment_ms"], eager["step_ms_min_median"][0])
+    assert lines["graph"]["ms_per_step"] >= 0.5 * floor
