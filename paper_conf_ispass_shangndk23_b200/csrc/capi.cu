@@ -69,6 +69,7 @@ struct Vec {
     int W = 1;     // elements per lane access
     int tile = 0;  // columns per launch (multiple of 32*W)
     bool deep = false;  // DRAM-bound gathers: the deep-gather instantiation (see below)
+    bool dram = false;  // a column tile's B slice exceeds half the L2 (gathers miss L2)
 };
 
 static int64_t l2_bytes() {
@@ -147,6 +148,7 @@ Vec choose_vec(int32_t K, int32_t dt, const void *B, int64_t ldb, const float *C
     // (profiles/r01/deep_gathers/).  MPS_DEEP=0/1 overrides.
     const char *ed = getenv("MPS_DEEP");
     const int kt = v.tile < K ? v.tile : K;
+    v.dram = b_rows > 0 && (double)b_rows * kt * eb > 0.5 * (double)l2_bytes();
     if (ed) v.deep = atoi(ed) != 0;
     else v.deep = b_rows > 0 && m > 0 && nnz >= 32 * m &&
                   (double)b_rows * kt * eb > 0.5 * (double)l2_bytes();
@@ -272,6 +274,16 @@ mps_status run_segments(mps::SegArgsT<IT> base, int32_t dt, int32_t K, const Vec
         int V, NR;
         tile_geometry(kt, v.W, &V, &NR);
         a.deep = v.deep && kt == 64 ? 1 : 0;
+        // next-batch L2 prefetch of B rows (bf16 dynamic kernels) where the tile's B slice
+        // exceeds half the L2; MPS_PF (read per call) 0/1 overrides
+        const char *ep = getenv("MPS_PF");
+        const int pfm = ep ? atoi(ep) : -1;
+        a.pf = pfm >= 0 ? pfm : (v.dram && dt == MPS_DT_BF16 ? 1 : 0);
+        {
+            int lines = (kt * eb + 127) / 128, sh = 0;
+            while ((1 << sh) < lines) ++sh;
+            a.pf_shift = sh;
+        }
         mps::SegArgsT<IT> seg_only = a;
         seg_only.mail.on = 0;
         MPS_CUDA(mps::launch_segments(fix == mps::FIX_CARRY ? seg_only : a, dt, v.W, V, NR, fix,

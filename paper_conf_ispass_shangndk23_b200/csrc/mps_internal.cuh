@@ -78,6 +78,9 @@ struct SegArgsT {
     unsigned *claim;     // dynamic segment claims: this column tile's counter in the caller's
                          // workspace, zero when the kernel starts (NULL: static assignment)
     int32_t deep;        // 1: deep-gather instantiation (fp32, 64-column tile, DRAM-bound B)
+    int32_t pf;          // 1: next-batch B rows into L2 while this batch is in flight
+                         // (dynamic bf16 instantiations; 0: off)
+    int32_t pf_shift;    // log2 of the 128-B lines per B row slice of this tile
     unsigned long long *wstat;  // Fig. 5 counters of what the kernel wrote (NULL: off):
                                 // [0] partial-row updates (atomic / carry record),
                                 // [1] empty partial start pieces whose add was elided,
@@ -314,6 +317,10 @@ template <> struct BVec<__nv_bfloat16, 1> {
     }
 };
 
+// The 128-B line holding p into L2 (LSU prefetch; no register, no scoreboard).
+__device__ __forceinline__ void prefetch_l2_line(const void *p) {
+    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(p));
+}
 // base + idx * stride as ONE mad.wide.u32 (IMAD.WIDE.U32 with a 64-bit addend).
 __device__ __forceinline__ const char *row_addr(const char *base, uint32_t idx, uint32_t stride) {
     uint64_t r;

@@ -54,6 +54,9 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_MINB_F32
 #define MPS_MINB_F32 3
 #endif
+#ifndef MPS_MINB_BF16_NARROW
+#define MPS_MINB_BF16_NARROW MPS_MINB_BF16   // bf16 lanes of < 16 B (W <= 4)
+#endif
 #ifndef MPS_UL_DIV
 #define MPS_UL_DIV 1
 #endif
@@ -92,13 +95,27 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_MINB_I64
 #define MPS_MINB_I64 3
 #endif
+// Threads per CTA of an instantiation: kBlock, or MPS_BF16_BLOCK for the 16-B bf16
+// gathers (experiment: smaller CTAs fit more warps per SM at ~96 registers)
+#ifndef MPS_BF16_BLOCK
+#define MPS_BF16_BLOCK 256
+#endif
+#ifndef MPS_BF16_SMALL_MINB
+#define MPS_BF16_SMALL_MINB 5
+#endif
+template <int W, typename TB, bool DEEP = false>
+__host__ __device__ constexpr int seg_block() {
+    return (sizeof(TB) == 2 && W >= 8 && !DEEP) ? MPS_BF16_BLOCK : kBlock;
+}
 template <int W, int V, typename TB, typename IT, bool DEEP = false>
-constexpr int seg_min_blocks() {
+__host__ __device__ constexpr int seg_min_blocks() {
     if constexpr (DEEP) return 2;
+    if constexpr (seg_block<W, TB, DEEP>() != kBlock) return MPS_BF16_SMALL_MINB;
     // int64 indices (NEXT-4): fp32 B measured best at 3 CTAs/SM with a few spills
     // (profiles/r01/next4), bf16 B keeps the int32 choice
     return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2
-           : (sizeof(TB) == 2 ? MPS_MINB_BF16 : (sizeof(IT) == 8 ? MPS_MINB_I64 : MPS_MINB_F32));
+           : (sizeof(TB) == 2 ? (W >= 8 ? MPS_MINB_BF16 : MPS_MINB_BF16_NARROW)
+                              : (sizeof(IT) == 8 ? MPS_MINB_I64 : MPS_MINB_F32));
 }
 
 // Gathers per lane per batch of a segment-kernel instantiation: ~4 KB of B rows in flight
@@ -116,16 +133,17 @@ __host__ __device__ constexpr int seg_ul() {
 }
 template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false,
           bool DYN = false>
-__global__ void __launch_bounds__(kBlock, (seg_min_blocks<W, V, TB, IT, DEEP>()))
+__global__ void __launch_bounds__((seg_block<W, TB, DEEP>()), (seg_min_blocks<W, V, TB, IT, DEEP>()))
 segment_kernel(const SegArgsT<IT> a) {
     using BV = BVec<TB, W>;
     using raw_t = typename BV::raw;
     static_assert(NR == 1 || V == 1, "several rows per instruction only for one slot");
     constexpr int LR = 32 / NR;                          // lanes per B row
-    constexpr int kWarps = kBlock / 32;
+    constexpr int kWarps = seg_block<W, TB, DEEP>() / 32;
     constexpr int UL = seg_ul<W, V, NR, TB, DEEP, DYN>();
     constexpr int U = UL * NR;                           // non-zeros per batch
     static_assert(kCH % U == 0, "chunk must hold whole batches");
+    constexpr bool kPF = DYN && sizeof(TB) == 2;         // next-batch L2 prefetch (bf16)
 
     __shared__ WarpStage stage[kWarps];
     __shared__ uint64_t bars[kWarps][2];
@@ -462,14 +480,16 @@ segment_kernel(const SegArgsT<IT> a) {
             int q = ys - cb;
             q = q > 0 ? (q / U) * U : 0;
             const int qend = min(kCH, ye - cb);
-            for (; q < qend; q += U) {
+            // issue(q, bv): the gathers of the batch at chunk offset q into bv;
+            // consume(q, bv): its FMAs and the rows it ends
+            auto issue = [&](const int q, raw_t (&bv)[UL][V]) {
                 const int j0 = cb + q;
-                raw_t bv[UL][V];
                 const bool full = j0 >= ys && j0 + U <= ye;
                 // my non-zeros of this batch: u = i*NR + grp (i < UL).  Column indices
                 // and values are read as broadcast 16-B LDS of 4 consecutive entries
-                // (NR <= 4) and each lane selects its own; branch-free: outside the
-                // segment the column index is clamped to 0 (a harmless in-bounds row).
+                // (NR <= MPS_BCAST_NR) and each lane selects its own, else per lane;
+                // branch-free: outside the segment the column index is clamped to 0 (a
+                // harmless in-bounds row).
                 uint32_t cid[UL];
                 if constexpr (NR <= MPS_BCAST_NR) {
 #pragma unroll
@@ -515,7 +535,28 @@ segment_kernel(const SegArgsT<IT> a) {
                                                     row_addr(bl[s], cid[i], ldb_bytes)), pol);
                     }
                 }
-
+                // bf16 B slices larger than L2: the B rows of the NEXT batch of this chunk
+                // go into L2 now (one LSU prefetch per lane, no registers held), so that
+                // batch's gathers wait for L2 hits instead of DRAM misses.  The bf16
+                // kernels hold only 16 warps per SM (128 registers): products bf16 -10%,
+                // R-MAT bf16 -3%; fp32 (24 warps) measured slower with it and does not
+                // carry the code (profiles/r03/prefetch.md)
+                if constexpr (kPF) {
+                    if (a.pf != 0) {
+                        const int qn = q + U;
+                        const int lines = 1 << a.pf_shift;
+                        for (int idx = lane; idx < U * lines; idx += 32) {
+                            const int t = idx >> a.pf_shift;
+                            if (qn + t < qend)
+                                prefetch_l2_line(row_addr(Bc, (uint32_t)sc[qn + t], ldb_bytes) +
+                                                 (idx & (lines - 1)) * 128);
+                        }
+                    }
+                }
+            };
+            auto consume = [&](const int q, const raw_t (&bv)[UL][V]) {
+                const int j0 = cb + q;
+                const bool full = j0 >= ys && j0 + U <= ye;
                 if (full && j0 + U <= rend) {
                     // fast path: U non-zeros of the current row, no checks
                     if constexpr (NR <= MPS_BCAST_NR) {
@@ -567,6 +608,11 @@ segment_kernel(const SegArgsT<IT> a) {
                         }
                     }
                 }
+            };
+            for (; q < qend; q += U) {
+                raw_t bv[UL][V];
+                issue(q, bv);
+                consume(q, bv);
             }
             ++ccount;
         }
@@ -604,7 +650,7 @@ static bool dynamic_claims() {
 // concurrent first calls from several host threads only repeat the same query.
 template <typename KFn>
 static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic, KFn kdyn,
-                                     int *out) {
+                                     int block, int *out) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -625,7 +671,7 @@ static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic,
         if (e != cudaSuccess) return e;
     }
     int bps = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kstatic, kBlock, 0);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kstatic, block, 0);
     if (e != cudaSuccess) return e;
     if (bps < 1) bps = 1;
     if (dev >= 0 && dev < 64) cache[dev].store(bps, std::memory_order_relaxed);
@@ -639,9 +685,10 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     auto kdy = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>;
     static std::atomic<int> occ_cache[64];      // per instantiation, per device
     int blocks_per_sm = 0;
-    cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, &blocks_per_sm);
+    constexpr int block = seg_block<W, TB, DEEP>();
+    cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, block, &blocks_per_sm);
     if (e != cudaSuccess) return e;
-    const int64_t warps_per_block = kBlock / 32;
+    const int64_t warps_per_block = block / 32;
     int64_t need = (a.P + warps_per_block - 1) / warps_per_block;
     const int64_t cap = (int64_t)blocks_per_sm * num_sms();
     const int64_t grid = need < cap ? need : cap;
@@ -665,7 +712,7 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     }();
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
-    cfg.blockDim = dim3(kBlock);
+    cfg.blockDim = dim3(block);
     cfg.dynamicSmemBytes = 0;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];

@@ -450,6 +450,30 @@ def test_deep_gather_variant(monkeypatch, fixup):
                 assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (K, dyn, cost)
 
 
+@pytest.mark.parametrize("fixup", ["atomic", "carry"])
+def test_bf16_next_batch_prefetch(monkeypatch, fixup):
+    """The bf16 dynamic kernels' next-batch L2 prefetch (on by rule where the tile's B
+    slice exceeds half the L2) forced on for a small graph with MPS_PF=1: it only moves
+    data into L2, so integer inputs stay bit-exact against the oracle for K = 64 (four
+    rows per instruction), 128 (two) and 256 (one 256-B slice per tile), batches that end
+    at chunk and segment edges, empty-row runs and a long row."""
+    monkeypatch.setenv("MPS_PF", "1")
+    monkeypatch.setenv("MPS_DYN", "1")
+    rs = np.random.RandomState(29)
+    rl = rs.randint(0, 12, size=20000).astype(np.int32)
+    rl[rs.rand(20000) < 0.4] = 0
+    rl[777] = 9000
+    g = G.random_csr(20000, 6000, rl, 37)
+    A = dev(g)
+    for K in (64, 128, 256):
+        B = G.dense_int(6000, K, seed=K + 1)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for cost in (5, 64, 0):
+            C = M.spmm(A, tB(B, torch.bfloat16), fixup=fixup, items_per_part=cost,
+                       min_parts=1 if cost else 0)
+            assert np.array_equal(C.cpu().numpy().astype(np.float64), ref), (K, cost)
+
+
 def test_carry_is_deterministic():
     g = G.workload("pubmed")
     B = tB(G.features("pubmed", 64))
