@@ -23,6 +23,7 @@
 #include <cuda_bf16.h>
 
 #include <cstdlib>
+#include <cstring>
 
 #include "mps_internal.cuh"
 
@@ -223,7 +224,8 @@ constexpr int kXpMaxStages = 8;
 
 __global__ void __launch_bounds__(kXpThreads, 1)
 xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
-                     const __grid_constant__ CUtensorMap map_w, int64_t n, int F, int N,
+                     const __grid_constant__ CUtensorMap map_w,
+                     const __grid_constant__ CUtensorMap map_b, int64_t n, int F, int N,
                      int stages, const XwDst dst, int64_t ldb, int staged, int nsplit,
                      int wstream) {
     // wstream = 1: W is NOT resident -- each ring stage carries the X chunk AND the
@@ -242,13 +244,16 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
     const uint32_t stage_bytes = a_bytes + (wstream ? wchunk : 0u);
     uint8_t *sW = base;
     uint8_t *sA = base + (wstream ? (size_t)0 : (size_t)nk * wchunk);
-    uint64_t *full = (uint64_t *)(sA + (size_t)stages * stage_bytes);
+    // staging tiles right after the ring (1024-B aligned: every stage is a multiple of
+    // 1 KB), barriers after them
+    uint8_t *stg = sA + (size_t)stages * stage_bytes;       // 8 warps x 32 rows x 64 B
+    uint64_t *full = (uint64_t *)(stg + 8 * 32 * 64);
     uint64_t *empty = full + kXpMaxStages;
     uint64_t *acc_full = empty + kXpMaxStages;              // [2]
     uint64_t *acc_empty = acc_full + 2;                     // [2]
     uint64_t *w_full = acc_empty + 2;
     uint32_t *tmem_slot = (uint32_t *)(w_full + 1);
-    uint8_t *stg = (uint8_t *)(acc_full + 64);              // 8 warps x 32 rows x 64 B
+
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int64_t ntiles = (n + kXwBM - 1) / kXwBM;
@@ -409,6 +414,36 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
                 // by (row >> 1) & 3 so that both the row-wise writes and the column-wise
                 // reads below hit 8 distinct 16-B bank groups per 8 lanes
                 uint32_t pk[16];
+                if (staged == 2) {
+                    // one destination, 32-column chunks: the 32 x 32 block leaves by a TMA
+                    // tensor store (the pattern is the tensor map's 64-B swizzle), issued by
+                    // one lane -- no per-lane address arithmetic or global stores
+#pragma unroll
+                    for (int j = 0; j < 16; ++j) {
+                        __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * j]),
+                                                                 __uint_as_float(v[2 * j + 1]));
+                        pk[j] = *reinterpret_cast<uint32_t *>(&h);
+                    }
+                    const uint32_t sb = smem_u32(wst);
+                    if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+                    __syncwarp();
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};"
+                                     :: "r"(sb + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)),
+                                        "r"(pk[4 * j]), "r"(pk[4 * j + 1]), "r"(pk[4 * j + 2]),
+                                        "r"(pk[4 * j + 3]) : "memory");
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    __syncwarp();
+                    if (lane == 0) {
+                        asm volatile(
+                            "cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];"
+                            :: "l"(&map_b), "r"(col_off + c0), "r"((int)(t * kXwBM) + q * 32), "r"(sb)
+                            : "memory");
+                        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+                    }
+                    continue;
+                }
 #pragma unroll
                 for (int j = 0; j < 16; ++j) {
                     __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * j]),
@@ -445,6 +480,8 @@ xw_persistent_kernel(const __grid_constant__ CUtensorMap map_x,
             }
         }
     }
+    if (staged == 2 && warp >= 2 && lane == 0)
+        asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // the TMA stores
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
     if (warp == 1)
@@ -480,6 +517,20 @@ bool make_map(CUtensorMap *map, const void *ptr, int64_t rows, int64_t cols, int
     return fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(ptr), dims, strides,
               box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// B (bf16 [rows][ld], cols used) as the destination of 32 x 32 TMA tensor stores, 64-B
+// swizzle (the persistent kernel's staging layout)
+bool make_store_map(CUtensorMap *map, const void *ptr, int64_t rows, int64_t cols, int64_t ld_elems) {
+    EncodeFn fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+    const cuuint64_t strides[1] = {(cuuint64_t)ld_elems * 2};
+    const cuuint32_t box[2] = {32, 32};
+    const cuuint32_t estr[2] = {1, 1};
+    return fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(ptr), dims, strides,
+              box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
+              CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 }  // namespace
@@ -527,6 +578,18 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
         const char *e = getenv("MPS_XW_STAGED");
         return e ? atoi(e) : 1;
     }();
+    // TMA-store epilogue (one destination, 32-column chunks); MPS_XW_TMA_STORE=0: per-lane
+    // global stores from the staging tiles (A/B)
+    static const int tma_store = [] {
+        const char *e = getenv("MPS_XW_TMA_STORE");
+        return e ? atoi(e) : 1;
+    }();
+    CUtensorMap mb;
+    memset(&mb, 0, sizeof(mb));
+    const bool can_tma_store = tma_store && staged && nd == 1 &&
+                               make_store_map(&mb, reinterpret_cast<const __nv_bfloat16 *>(dsts[0]) + row_offset * ldb,
+                                              n, N, ldb);
+    auto staged_mode = [&](int nh) { return (can_tma_store && nh % 32 == 0) ? 2 : staged; };
     const size_t xw_budget = 227u << 10, xw_fixed = 1024 + 512 + 8 * 32 * 64;
     auto set_persist_attr = [&]() -> cudaError_t {
         // function attributes are per device: set once for each
@@ -558,7 +621,7 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
         int64_t grid = (int64_t)num_sms() * per_sm;
         if (grid > ntiles) grid = ntiles;
         xw_persistent_kernel<<<(unsigned)grid, kXpThreads, smem, s>>>(
-            mx, mw, n, (int)F, N, stages, dst, ldb, staged, 1, 1);
+            mx, mw, mb, n, (int)F, N, stages, dst, ldb, staged_mode(N), 1, 1);
         return cudaGetLastError();
     };
     if (persist && wstream_env == 1) return launch_wstream();
@@ -570,7 +633,7 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
         // shared memory) or else one; slices only when W does not fit at all.
         const int nkp = (int)((F + kXwBK - 1) / kXwBK);
         const size_t a_bytes = (size_t)kXwBM * kXwBK * 2;
-        const size_t fixed = 1024 + 512 + 8 * 32 * 64;      // align, barriers, staging
+        const size_t fixed = xw_fixed;                      // align, barriers, staging
         const size_t budget = 227u << 10, half_budget = 113u << 10;
         auto wb = [&](int nh) { return (size_t)nkp * nh * kXwBK * 2; };
         int nh = 0, per_sm = 0;
@@ -605,7 +668,8 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
             if (grid > ntiles * nsplit) grid = ntiles * nsplit;
             if (grid < nsplit) grid = nsplit;
             xw_persistent_kernel<<<(unsigned)grid, kXpThreads, smem, s>>>(
-                mx, nh == N ? mw : mws, n, (int)F, nh, stages, dst, ldb, staged, nsplit, 0);
+                mx, nh == N ? mw : mws, mb, n, (int)F, nh, stages, dst, ldb, staged_mode(nh),
+                nsplit, 0);
             return cudaGetLastError();
         }
         // W does not fit in shared memory: stream it through the ring with X (the
