@@ -657,6 +657,11 @@ static cudaError_t launch_xw(const void *X, int64_t n, int64_t F, int64_t ldx, c
             const int nsplit = N / nh;
             int stages = (int)(((per_sm == 2 ? half_budget : budget) - fixed - wb(nh)) / a_bytes);
             stages = stages > max_stages ? max_stages : stages;
+            // B at least as wide as X (N >= F: as many bytes written as read): a shallow
+            // 3-stage X ring measured fastest (big-F 1M x 256 x 256: 3 stages 0.172 ms,
+            // 4: 0.177, 5: 0.188; products neutral; profiles/r03/xw_tma_store.md), the
+            // wide-F shapes want every stage (Reddit F=602: 8 stages 0.071, 3: 0.083)
+            if (N >= F && stages > 3 && max_stages == kXpMaxStages) stages = 3;
             stages = stages < 2 ? 2 : stages;
             const size_t smem = fixed + wb(nh) + (size_t)stages * a_bytes;
             cudaError_t ea = set_persist_attr();
