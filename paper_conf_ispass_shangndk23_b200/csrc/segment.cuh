@@ -89,6 +89,9 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #ifndef MPS_EMPTY_RUNS
 #define MPS_EMPTY_RUNS -1
 #endif
+#ifndef MPS_SLOW_VL_REG
+#define MPS_SLOW_VL_REG 1
+#endif
 #ifndef MPS_SLOW_PARTS
 #define MPS_SLOW_PARTS 0     // 0: the measured rule below (2 parts for >= 32-non-zero batches)
 #endif
@@ -96,21 +99,25 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #define MPS_MINB_I64 3
 #endif
 // Threads per CTA of an instantiation: kBlock, or MPS_BF16_BLOCK for the 16-B bf16
-// gathers (experiment: smaller CTAs fit more warps per SM at ~96 registers)
+// gathers with >= 4 rows per warp instruction (int32 indices): 5 CTAs of 4 warps at 96
+// registers (slow-path values re-read from shared memory, no spills) hold 20 warps per
+// SM instead of 16 -- R-MAT bf16 K=64 -3.4%, products bf16 K=64 -3.0%, Reddit bf16 K=64
+// -0.3% (profiles/r03/prefetch.md); 256 restores 2 x 8 warps at 128 registers
 #ifndef MPS_BF16_BLOCK
-#define MPS_BF16_BLOCK 256
+#define MPS_BF16_BLOCK 128
 #endif
 #ifndef MPS_BF16_SMALL_MINB
 #define MPS_BF16_SMALL_MINB 5
 #endif
-template <int W, typename TB, bool DEEP = false>
+template <int W, int NR, typename TB, typename IT, bool DEEP = false>
 __host__ __device__ constexpr int seg_block() {
-    return (sizeof(TB) == 2 && W >= 8 && !DEEP) ? MPS_BF16_BLOCK : kBlock;
+    return (sizeof(TB) == 2 && sizeof(IT) == 4 && W >= 8 && NR >= 4 && !DEEP) ? MPS_BF16_BLOCK
+                                                                              : kBlock;
 }
-template <int W, int V, typename TB, typename IT, bool DEEP = false>
+template <int W, int V, int NR, typename TB, typename IT, bool DEEP = false>
 __host__ __device__ constexpr int seg_min_blocks() {
     if constexpr (DEEP) return 2;
-    if constexpr (seg_block<W, TB, DEEP>() != kBlock) return MPS_BF16_SMALL_MINB;
+    if constexpr (seg_block<W, NR, TB, IT, DEEP>() != kBlock) return MPS_BF16_SMALL_MINB;
     // int64 indices (NEXT-4): fp32 B measured best at 3 CTAs/SM with a few spills
     // (profiles/r01/next4), bf16 B keeps the int32 choice
     return (V * ((W * (int)sizeof(TB) + 3) / 4) > 8) ? 2
@@ -133,13 +140,17 @@ __host__ __device__ constexpr int seg_ul() {
 }
 template <int W, int V, int NR, typename TB, int FIX, typename IT, bool DEEP = false,
           bool DYN = false>
-__global__ void __launch_bounds__((seg_block<W, TB, DEEP>()), (seg_min_blocks<W, V, TB, IT, DEEP>()))
+__global__ void __launch_bounds__((seg_block<W, NR, TB, IT, DEEP>()),
+                                  (seg_min_blocks<W, V, NR, TB, IT, DEEP>()))
 segment_kernel(const SegArgsT<IT> a) {
     using BV = BVec<TB, W>;
     using raw_t = typename BV::raw;
     static_assert(NR == 1 || V == 1, "several rows per instruction only for one slot");
     constexpr int LR = 32 / NR;                          // lanes per B row
-    constexpr int kWarps = seg_block<W, TB, DEEP>() / 32;
+    constexpr int kWarps = seg_block<W, NR, TB, IT, DEEP>() / 32;
+    // slow-path values held in registers, or re-read from shared memory in each pass (the
+    // small-CTA bf16 instantiations, to stay within their register budget without spills)
+    constexpr bool kVlReg = MPS_SLOW_VL_REG && seg_block<W, NR, TB, IT, DEEP>() == kBlock;
     constexpr int UL = seg_ul<W, V, NR, TB, DEEP, DYN>();
     constexpr int U = UL * NR;                           // non-zeros per batch
     static_assert(kCH % U == 0, "chunk must hold whole batches");
@@ -576,9 +587,13 @@ segment_kernel(const SegArgsT<IT> a) {
                     // slow path: the batch crosses row ends (or the segment's edges).
                     // One pass per row intersecting the batch: predicated FMAs for the
                     // non-zeros of the current row, then settle the row.
+                    // values in registers for the passes (MPS_SLOW_VL_REG=1), or re-read
+                    // from shared memory inside each pass (0: fewer live registers)
                     float vl[UL];
+                    if constexpr (kVlReg) {
 #pragma unroll
-                    for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
+                        for (int i = 0; i < UL; ++i) vl[i] = sv[q + i * NR + grp];
+                    }
                     // The batch is settled in SP parts of UL/SP entries each; a part's
                     // passes predicate only its own entries, so a row end costs UL/SP
                     // FMA groups instead of UL (MPS_SLOW_PARTS, measured in
@@ -602,7 +617,8 @@ segment_kernel(const SegArgsT<IT> a) {
 #pragma unroll
                             for (int i = h * ULP; i < (h + 1) * ULP; ++i) {
                                 const int j = j0 + i * NR + grp;
-                                if (j >= jc && j < lim) fma_row(vl[i], bv[i]);
+                                if (j >= jc && j < lim)
+                                    fma_row(kVlReg ? vl[i] : sv[q + i * NR + grp], bv[i]);
                             }
                             jc = lim;
                         }
@@ -685,7 +701,7 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     auto kdy = segment_kernel<W, V, NR, TB, FIX, IT, DEEP, true>;
     static std::atomic<int> occ_cache[64];      // per instantiation, per device
     int blocks_per_sm = 0;
-    constexpr int block = seg_block<W, TB, DEEP>();
+    constexpr int block = seg_block<W, NR, TB, IT, DEEP>();
     cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, block, &blocks_per_sm);
     if (e != cudaSuccess) return e;
     const int64_t warps_per_block = block / 32;

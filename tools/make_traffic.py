@@ -5,23 +5,25 @@ Usage: python tools/make_traffic.py TAG [dir]   (reads DIR/ncu_TAG_<wl>_k<K>_raw
 import csv, json, os, sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-TILES = {"reddit-k64": 1, "reddit-k256": 4, "products-k128": 2, "rmat-k64": 1}
+# (workload-kK, B dtype) -> column tiles per step (bf16: 128-column tiles of 256 B)
+TILES = {("reddit-k64", "f32"): 1, ("reddit-k256", "f32"): 4, ("products-k128", "f32"): 2,
+         ("rmat-k64", "f32"): 1, ("products-k128", "bf16"): 1}
 UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
 
 
 def main(tag, d):
     out = {}
     units = {}
-    for wl, tiles in TILES.items():
+    for (wl, dt), tiles in TILES.items():
         name, k = wl.split("-k")
-        path = os.path.join(d, "ncu_%s_%s_k%s_raw.csv" % (tag, name, k))
+        path = os.path.join(d, "ncu_%s_%s_k%s%s_raw.csv" % (tag, name, k, "" if dt == "f32" else "_" + dt))
         if not os.path.exists(path):
             continue
         rows = list(csv.reader(open(path)))
         hdr, un, val = rows[0], rows[1], rows[2]
         get = lambda m: float(val[hdr.index(m)])
         b = lambda m: get(m) * UNIT[un[hdr.index(m)]]
-        key = "%s-f32-atomic" % wl
+        key = "%s-%s-atomic" % (wl, dt)
         out[key] = int(round((b("dram__bytes_read.sum") + b("dram__bytes_write.sum")) * tiles))
         units[key] = {
             "lts_throughput_pct": round(get("lts__throughput.avg.pct_of_peak_sustained_elapsed"), 1),

@@ -50,6 +50,20 @@ def run():
                 if not np.array_equal(C.cpu().numpy().astype(np.float64), ref):
                     print("MISMATCH dynamic claims", K, dt, fixup)
                     bad += 1
+    # bf16 next-batch L2 prefetch forced on (dynamic claims; 4, 2 and 1 rows per
+    # instruction)
+    os.environ["MPS_PF"] = "1"
+    for K in (64, 128, 256):
+        B = G.dense_int(2000, K, seed=K + 5)
+        ref = O.csr_spmm_f64(g.row_ptr, g.col_idx, g.val, B, want_bound=False)
+        for fixup in ("atomic", "carry"):
+            C = M.spmm(A, torch.from_numpy(B).cuda().to(torch.bfloat16), fixup=fixup,
+                       items_per_part=2, min_parts=1)
+            torch.cuda.synchronize()
+            if not np.array_equal(C.cpu().numpy().astype(np.float64), ref):
+                print("MISMATCH bf16 prefetch", K, fixup)
+                bad += 1
+    del os.environ["MPS_PF"]
     # deep-gather instantiation forced on (fp32, 64-column tiles), static and dynamic
     os.environ["MPS_DEEP"] = "1"
     os.environ["MPS_TILE"] = "64"
@@ -119,6 +133,14 @@ def run():
     torch.cuda.synchronize()
     if not all(torch.equal(t.double().cpu(), ref) for t in reps):
         print("MISMATCH xw bcast")
+        bad += 1
+    # B as wide as X (N >= F): the 3-stage ring, TMA-store epilogue, partial last tile
+    n, F, N = 1000, 64, 128
+    X = torch.randint(-1, 2, (n, F), generator=gen).to(torch.bfloat16)
+    W = torch.randint(-1, 2, (F, N), generator=gen).to(torch.bfloat16)
+    if not torch.equal(M.xw_bf16(X.cuda(), W.t().contiguous().cuda()).double().cpu(),
+                       X.double() @ W.double()):
+        print("MISMATCH xw N >= F")
         bad += 1
     print("sanitize cases done, mismatches:", bad)
     return bad
