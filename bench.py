@@ -770,6 +770,26 @@ def main():
                                               "hbm_peak": seg_gbs / hbm_peak}
                 roof.update({"peak": seg_bytes / (t_rep * 1e-3) / 1e9, "frac": t_rep / t_seg,
                              "peak_source": "gather replay of this workload (roofline.attainable)"})
+                # the same replay at the fp32 kernel's own register-resident depth (3 CTAs
+                # x 8 warps, 8 x 16-B gathers per lane; the deep-gather kernel: 2 CTAs, 16):
+                # what the gather stream alone takes with the bytes in flight the kernel
+                # can hold -- a diagnostic beside the attainable replay, not the peak
+                if b_elt == 4 and row_bytes == 256:
+                    deep = g.nnz >= 32 * g.n and g.n * row_bytes > 0.5 * l2
+                    psm, ul = (2, 0) if deep else (3, 8)
+                    sms, sby = ctypes.c_float(), ctypes.c_double()
+                    rc2 = gr.gather_replay_cfg(_p(A.col_idx), ctypes.c_int64(g.nnz), _p(Bd),
+                                               ctypes.c_int32(row_bytes), ctypes.c_int64(K * b_elt),
+                                               ctypes.c_int32(3), ctypes.c_int32(psm),
+                                               ctypes.c_int32(ul), ctypes.byref(sms),
+                                               ctypes.byref(sby))
+                    torch.cuda.synchronize(dev)
+                    if rc2 == 0 and sms.value > 0:
+                        roof["attainable"]["same_depth"] = {
+                            "what": "the same replay with the kernel's bytes in flight: %d CTAs "
+                                    "x 8 warps per SM, %d x 16-B gathers per lane" % (
+                                        psm, ul or 16),
+                            "replay_ms": sms.value * tiles, "frac": sms.value * tiles / t_seg}
         except Exception as e:  # pragma: no cover
             roof["attainable_error"] = str(e)[:200]
 

@@ -18,14 +18,15 @@ __device__ __forceinline__ uint4 ldg_b(const void *p, uint64_t pol) {
 }
 
 // row_bytes in {64, 128, 256, 512}: LR = row_bytes/16 lanes per row, NR = 32/LR rows per
-// warp instruction; a batch = 32 non-zeros = 32/NR instructions, 16 in flight per lane
-// for 256-B rows (UL = 32/NR).
-template <int LR>
+// warp instruction; a batch = UL*NR non-zeros, UL gathers in flight per lane (UL = 32/NR
+// by default: 16 for 256-B rows; ULC caps it, e.g. 8 = the segment kernel's own depth).
+template <int LR, int ULC = 32>
 __global__ void __launch_bounds__(256) replay_kernel(const int32_t *__restrict__ col, int64_t nnz,
                                                      const char *__restrict__ B, int64_t ldb_bytes,
                                                      int64_t per_warp, uint32_t *sink) {
     constexpr int NR = 32 / LR;
-    constexpr int UL = 32 / NR;
+    constexpr int UL = (32 / NR) < ULC ? (32 / NR) : ULC;
+    constexpr int U = UL * NR;
     const int lane = threadIdx.x & 31, grp = lane / LR, lr = lane % LR;
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     int64_t j0 = warp * per_warp;
@@ -33,9 +34,9 @@ __global__ void __launch_bounds__(256) replay_kernel(const int32_t *__restrict__
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
     uint32_t acc = 0;
-    for (; j0 < j1; j0 += 32) {
+    for (; j0 < j1; j0 += U) {
         const int64_t j = j0 + lane;
-        const int c = j < j1 ? __ldg(col + j) : 0;
+        const int c = (lane < U && j < j1) ? __ldg(col + j) : 0;
         uint4 v[UL];
 #pragma unroll
         for (int i = 0; i < UL; ++i) {
@@ -49,10 +50,25 @@ __global__ void __launch_bounds__(256) replay_kernel(const int32_t *__restrict__
 }
 }  // namespace
 
-// Gathers rows col[0..nnz) of B (row_bytes of each row, stride ldb_bytes), returns the
-// best time over a few grid shapes (ms) and the bytes it moved (gathered rows + col).
-extern "C" int gather_replay(const int32_t *col, int64_t nnz, const void *B, int32_t row_bytes,
-                             int64_t ldb_bytes, int32_t reps, float *best_ms, double *bytes) {
+template <int ULC>
+static int replay_launch(int row_bytes, int64_t grid, const int32_t *col, int64_t nnz,
+                         const void *B, int64_t ldb_bytes, int64_t per, uint32_t *sink) {
+    switch (row_bytes) {
+    case 64: replay_kernel<4, ULC><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
+    case 128: replay_kernel<8, ULC><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
+    case 256: replay_kernel<16, ULC><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
+    case 512: replay_kernel<32, ULC><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
+    default: return 3;
+    }
+    return 0;
+}
+
+// Gathers rows col[0..nnz) of B (row_bytes of each row, stride ldb_bytes) with the given
+// resident CTAs (8 warps) per SM (0: best of 3, 4, 6) and gathers per lane (ul: 0 = 16
+// for 256-B rows, or 8); returns the best time (ms) and the bytes it moved.
+extern "C" int gather_replay_cfg(const int32_t *col, int64_t nnz, const void *B, int32_t row_bytes,
+                                 int64_t ldb_bytes, int32_t reps, int32_t per_sm_only, int32_t ul,
+                                 float *best_ms, double *bytes) {
     int dev = 0, sms = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -68,34 +84,40 @@ extern "C" int gather_replay(const int32_t *col, int64_t nnz, const void *B, int
     cudaEventCreate(&e1);
     float best = 1e30f;
     const int per_sm[3] = {3, 4, 6};
-    for (int c = 0; c < 3; ++c) {
-        const int64_t warps = (int64_t)sms * per_sm[c] * 8;
+    int rc = 0;
+    for (int c = 0; c < 3 && rc == 0; ++c) {
+        const int psm = per_sm_only > 0 ? per_sm_only : per_sm[c];
+        const int64_t warps = (int64_t)sms * psm * 8;
         int64_t per = (nnz + warps - 1) / warps;
         per = (per + 31) / 32 * 32;
         const int64_t nw = (nnz + per - 1) / per;
         const int64_t grid = (nw + 7) / 8;
-        for (int r = 0; r < reps + 1; ++r) {
+        for (int r = 0; r < reps + 1 && rc == 0; ++r) {
             cudaMemsetAsync(flush, r & 1, (size_t)l2 * 2);
             cudaEventRecord(e0);
-            switch (row_bytes) {
-            case 64: replay_kernel<4><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
-            case 128: replay_kernel<8><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
-            case 256: replay_kernel<16><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
-            case 512: replay_kernel<32><<<(unsigned)grid, 256>>>(col, nnz, (const char *)B, ldb_bytes, per, sink); break;
-            default: return 3;
-            }
+            rc = ul == 8 ? replay_launch<8>(row_bytes, grid, col, nnz, B, ldb_bytes, per, sink)
+                         : replay_launch<32>(row_bytes, grid, col, nnz, B, ldb_bytes, per, sink);
             cudaEventRecord(e1);
             cudaEventSynchronize(e1);
             float t = 0.f;
             cudaEventElapsedTime(&t, e0, e1);
             if (r > 0 && t < best) best = t;       // first launch: warm-up
         }
+        if (per_sm_only > 0) break;
     }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     cudaFree(sink);
     cudaFree(flush);
+    if (rc) return rc;
     *best_ms = best;
     *bytes = (double)nnz * row_bytes + (double)nnz * 4;
     return cudaGetLastError() == cudaSuccess ? 0 : 2;
+}
+
+// The attainable replay of bench.py's roofline: best of 3 / 4 / 6 CTAs per SM, 16 gathers
+// of 16 B in flight per lane for 256-B rows.
+extern "C" int gather_replay(const int32_t *col, int64_t nnz, const void *B, int32_t row_bytes,
+                             int64_t ldb_bytes, int32_t reps, float *best_ms, double *bytes) {
+    return gather_replay_cfg(col, nnz, B, row_bytes, ldb_bytes, reps, 0, 0, best_ms, bytes);
 }
