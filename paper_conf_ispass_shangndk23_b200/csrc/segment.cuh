@@ -26,8 +26,12 @@
 
 namespace mps {
 
+// non-zeros per staged col/val chunk (per warp; two chunks in flight): 512 = 8 KB per
+// warp of dynamic shared memory (192 KB for 3 x 8 fp32 warps per SM).  Measured against
+// 256 (profiles/r03/chunk.md): R-MAT -1.3%, Reddit -0.5%, products -0.9%, bf16 Reddit -4%,
+// bf16 R-MAT -1.8%; 128 was slower everywhere
 #ifndef MPS_CHUNK
-#define MPS_CHUNK 256
+#define MPS_CHUNK 512
 #endif
 constexpr int kCH = MPS_CHUNK;     // non-zeros per staged chunk (per warp)
 constexpr int kSegMinBlocks = 3;   // 24 resident warps/SM (<= 80 registers)
@@ -156,7 +160,10 @@ segment_kernel(const SegArgsT<IT> a) {
     static_assert(kCH % U == 0, "chunk must hold whole batches");
     constexpr bool kPF = DYN && sizeof(TB) == 2;         // next-batch L2 prefetch (bf16)
 
-    __shared__ WarpStage stage[kWarps];
+    // per-warp col/val staging in dynamic shared memory (kWarps x sizeof(WarpStage), set
+    // by the launcher; > 48 KB for large chunks)
+    extern __shared__ __align__(16) uint8_t seg_dsmem[];
+    WarpStage *stage = reinterpret_cast<WarpStage *>(seg_dsmem);
     __shared__ uint64_t bars[kWarps][2];
 
     const int warp = threadIdx.x >> 5;
@@ -666,7 +673,7 @@ static bool dynamic_claims() {
 // concurrent first calls from several host threads only repeat the same query.
 template <typename KFn>
 static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic, KFn kdyn,
-                                     int block, int *out) {
+                                     int block, size_t dsmem, int *out) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -686,8 +693,14 @@ static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic,
             e = cudaFuncSetAttribute(kdyn, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
         if (e != cudaSuccess) return e;
     }
+    if (dsmem > (48u << 10)) {
+        e = cudaFuncSetAttribute(kstatic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(kdyn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
+        if (e != cudaSuccess) return e;
+    }
     int bps = 0;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kstatic, block, 0);
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, kstatic, block, dsmem);
     if (e != cudaSuccess) return e;
     if (bps < 1) bps = 1;
     if (dev >= 0 && dev < 64) cache[dev].store(bps, std::memory_order_relaxed);
@@ -702,7 +715,8 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     static std::atomic<int> occ_cache[64];      // per instantiation, per device
     int blocks_per_sm = 0;
     constexpr int block = seg_block<W, NR, TB, IT, DEEP>();
-    cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, block, &blocks_per_sm);
+    constexpr size_t dsmem = (size_t)(block / 32) * sizeof(WarpStage);
+    cudaError_t e = seg_blocks_per_sm(occ_cache, kst, kdy, block, dsmem, &blocks_per_sm);
     if (e != cudaSuccess) return e;
     const int64_t warps_per_block = block / 32;
     int64_t need = (a.P + warps_per_block - 1) / warps_per_block;
@@ -729,7 +743,7 @@ static cudaError_t launch_seg(const SegArgsT<IT> &a, cudaStream_t s) {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = dim3(block);
-    cfg.dynamicSmemBytes = 0;
+    cfg.dynamicSmemBytes = dsmem;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
