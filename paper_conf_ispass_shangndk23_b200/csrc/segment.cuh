@@ -154,7 +154,8 @@ segment_kernel(const SegArgsT<IT> a) {
     constexpr int kWarps = seg_block<W, NR, TB, IT, DEEP>() / 32;
     // slow-path values held in registers, or re-read from shared memory in each pass (the
     // small-CTA bf16 instantiations, to stay within their register budget without spills)
-    constexpr bool kVlReg = MPS_SLOW_VL_REG && seg_block<W, NR, TB, IT, DEEP>() == kBlock;
+    constexpr bool kVlReg = MPS_SLOW_VL_REG && seg_block<W, NR, TB, IT, DEEP>() == kBlock &&
+                            !(MPS_MINB_F32 > 3 && sizeof(TB) == 4);
     constexpr int UL = seg_ul<W, V, NR, TB, DEEP, DYN>();
     constexpr int U = UL * NR;                           // non-zeros per batch
     static_assert(kCH % U == 0, "chunk must hold whole batches");
@@ -693,7 +694,7 @@ static cudaError_t seg_blocks_per_sm(std::atomic<int> (&cache)[64], KFn kstatic,
             e = cudaFuncSetAttribute(kdyn, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
         if (e != cudaSuccess) return e;
     }
-    if (dsmem > (48u << 10)) {
+    if (dsmem > 0) {   // (the 48-KB default limit counts the static barriers too)
         e = cudaFuncSetAttribute(kstatic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
         if (e == cudaSuccess)
             e = cudaFuncSetAttribute(kdyn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem);
