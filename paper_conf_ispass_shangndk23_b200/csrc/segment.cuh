@@ -103,20 +103,25 @@ __device__ __forceinline__ float pick4f(const float4 &v, int e) {
 #define MPS_MINB_I64 3
 #endif
 // Threads per CTA of an instantiation: kBlock, or MPS_BF16_BLOCK for the 16-B bf16
-// gathers with >= 4 rows per warp instruction (int32 indices): 5 CTAs of 4 warps at 96
-// registers (slow-path values re-read from shared memory, no spills) hold 20 warps per
-// SM instead of 16 -- R-MAT bf16 K=64 -3.4%, products bf16 K=64 -3.0%, Reddit bf16 K=64
-// -0.3% (profiles/r03/prefetch.md); 256 restores 2 x 8 warps at 128 registers
+// gathers with >= 2 rows per warp instruction (int32 indices): 5 CTAs of 4 warps at 96
+// registers (slow-path values re-read from shared memory, slow path in two parts, no
+// spills) hold 20 warps per SM instead of 16 -- R-MAT bf16 K=64 -3.4%, products bf16
+// K=64 -3.0%, Reddit bf16 K=64 -0.3%; two rows per instruction (256-B bf16 rows):
+// products K=128 -3.2%, Reddit K=256 -7.6%, R-MAT K=128 -7.4% (profiles/r03/prefetch.md);
+// 256 restores 2 x 8 warps at 128 registers
 #ifndef MPS_BF16_BLOCK
 #define MPS_BF16_BLOCK 128
+#endif
+#ifndef MPS_BF16_SMALL_MINNR
+#define MPS_BF16_SMALL_MINNR 2   // rows per warp instruction from which the small CTAs apply
 #endif
 #ifndef MPS_BF16_SMALL_MINB
 #define MPS_BF16_SMALL_MINB 5
 #endif
 template <int W, int NR, typename TB, typename IT, bool DEEP = false>
 __host__ __device__ constexpr int seg_block() {
-    return (sizeof(TB) == 2 && sizeof(IT) == 4 && W >= 8 && NR >= 4 && !DEEP) ? MPS_BF16_BLOCK
-                                                                              : kBlock;
+    return (sizeof(TB) == 2 && sizeof(IT) == 4 && W >= 8 && NR >= MPS_BF16_SMALL_MINNR && !DEEP)
+               ? MPS_BF16_BLOCK : kBlock;
 }
 template <int W, int V, int NR, typename TB, typename IT, bool DEEP = false>
 __host__ __device__ constexpr int seg_min_blocks() {
@@ -608,7 +613,9 @@ segment_kernel(const SegArgsT<IT> a) {
                     // profiles/r02/slow_steps.md)
                     // (default: two parts for batches of >= 32 non-zeros -- bf16 K=64 /
                     // fp32 K=32 -- where they measured 4-6% faster; one part otherwise)
-                    constexpr int SP0 = MPS_SLOW_PARTS > 0 ? MPS_SLOW_PARTS : (U >= 32 ? 2 : 1);
+                    // (and two parts in the small-CTA bf16 kernels: fewer live registers)
+                    constexpr int SP0 = MPS_SLOW_PARTS > 0 ? MPS_SLOW_PARTS
+                                        : ((U >= 32 || !kVlReg) ? 2 : 1);
                     constexpr int SP = (UL % SP0 == 0) ? SP0 : 1;
                     constexpr int ULP = UL / SP;
                     int jc = j0 > ys ? j0 : ys;                  // next non-zero to consume
