@@ -94,3 +94,35 @@ def test_xw_streamed_w_forced_exact():
                         "exact_small_integers"], env=env, capture_output=True, text=True,
                        timeout=600, cwd=root)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+
+
+def test_xw_strided_output_keeps_padding():
+    """The TMA-store epilogue writes B through a tensor map of the output's own row stride:
+    a strided `out` (ldb > N) gets exactly its N columns, the padding keeps its sentinel,
+    rows past a ragged last tile are not written (N = 64: whole 32-column chunks)."""
+    g = torch.Generator(device="cpu").manual_seed(5)
+    n, F, N, ldb = 1000 + 33, 64, 64, 96
+    X = torch.randint(-1, 2, (n, F), generator=g).to(torch.bfloat16).cuda()
+    W = torch.randint(-1, 2, (F, N), generator=g).to(torch.bfloat16).cuda()
+    full = torch.full((n + 5, ldb), 7.0, dtype=torch.bfloat16, device="cuda")
+    out = full[:n, :N]
+    M.xw_bf16(X, W.t().contiguous(), out=out)
+    ref = torch.from_numpy(O.xw_f64(X.float().cpu().numpy(), W.float().cpu().numpy()))
+    assert torch.equal(out.double().cpu(), ref)
+    assert torch.all(full[:, N:] == 7.0) and torch.all(full[n:] == 7.0)
+
+
+@pytest.mark.parametrize("env", [{"MPS_XW_TMA_STORE": "0"}, {"MPS_XW_SPLIT": "2"},
+                                 {"MPS_XW_STAGES": "8"}])
+def test_xw_epilogue_variants_exact(env):
+    """The per-lane store epilogue (MPS_XW_TMA_STORE=0), column slices on consecutive CTAs
+    (MPS_XW_SPLIT=2: TMA stores at a column offset) and the full-depth ring for N >= F
+    (MPS_XW_STAGES=8): the small-integer shapes stay bit-exact against O9 (the knobs are
+    read once per process: run in a subprocess)."""
+    import os, subprocess, sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-p", "no:cacheprovider",
+                        os.path.join(root, "tests", "test_gpu_xw.py"), "-k",
+                        "exact_small_integers or strided_output"], env=dict(os.environ, **env),
+                       capture_output=True, text=True, timeout=900, cwd=root)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
