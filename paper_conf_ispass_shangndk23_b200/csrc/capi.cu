@@ -51,13 +51,16 @@ inline int elt_bytes(int32_t dt) { return dt == MPS_DT_BF16 ? 2 : 4; }
 //   cost = max(64, min(clamp(next_pow2(4*ceil(nnz/m)), 512, 2048),
 //                      pow2_floor(M / (1.5 * resident_warps))))
 // (geomean 0.974 of the per-graph best on Table II, 0.998 on Reddit/products/R-MAT).
+// Resident warps: 24 per SM for fp32, 20 for bf16 (the 128-thread bf16 CTAs of round 2's
+// second session; with 16 the bf16 Table-II score fell to 0.933, with 20 it is 0.966 --
+// profiles/r03/sensitivity.md; the BASELINE graphs' costs do not change).
 int64_t default_cost(int64_t m, int64_t nnz, int32_t K, int32_t dt) {
     (void)K;
     const int64_t avg = m > 0 ? (nnz + m - 1) / m : 1;
     int64_t deg = 1;
     while (deg < 4 * avg) deg <<= 1;
     deg = deg < 512 ? 512 : (deg > 2048 ? 2048 : deg);
-    const int64_t resident = (int64_t)mps::num_sms() * (dt == MPS_DT_BF16 ? 16 : 24);
+    const int64_t resident = (int64_t)mps::num_sms() * (dt == MPS_DT_BF16 ? 20 : 24);
     const double target = (double)(m + nnz) / (1.5 * (double)resident);
     int64_t cap = 1;
     while ((double)(cap * 2) <= target) cap <<= 1;
